@@ -1,0 +1,168 @@
+/*
+ * sat.h -- libsat: single-pass summed area tables on NVIDIA B200 (sm_100a).  C ABI.
+ *
+ * PAPER.md = /root/reference/PAPER.md (Emoto et al., "An Optimal Parallel Algorithm for
+ * Computing the Summed Area Table on the GPU", IPDPSW 2018), cited as P:<line>.
+ *
+ * The operation (Sec. I.A; restated P:132, Sec. III):
+ *     dst[i][j] = sum_{0<=i'<=i, 0<=j'<=j} src[i'][j']        0 <= i < rows, 0 <= j < cols
+ * for a row-major matrix "stored in the global memory of the GPU", the result "written in the
+ * global memory" (Sec. I.C), element [i][j] at offset i*pitch + j (pitch >= cols is
+ * reading R3 of DESIGN.md).  It is computed in ONE kernel pass that reads every element once and
+ * writes every element once (the 1R1W-SKSS-LB method of Sec. IV: a dynamic tile
+ * counter, per-tile published aggregates and look-back), re-designed for sm_100a.
+ *
+ * General rules for every entry point:
+ *   - extern "C", never throws, returns sat_status_t; on failure sat_last_error_detail() gives a
+ *     thread-local human-readable detail (CUDA/NCCL error text included).
+ *   - Pointers documented as "device" must point to memory of the CURRENT CUDA device (the device
+ *     of `stream`); "host" pointers are ordinary (pageable or pinned) host memory.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Device-pointer
+ *     calls are stream-ordered and asynchronous (no host synchronisation).
+ *   - Sizes are int64_t element counts.  rows == 0 or cols == 0 is a no-op returning SAT_OK.
+ *     Negative sizes or pitch < cols return SAT_ERR_INVALID_VALUE.
+ *   - Pointers not aligned to the 4-byte element size return SAT_ERR_MISALIGNED.  16-byte alignment
+ *     of both pointers and of pitch*4 selects the TMA fast path; otherwise a slower path is used.
+ *   - Pad elements [cols, pitch) of every row of dst are never written.
+ *   - src == dst (in place) is allowed; any other overlap returns SAT_ERR_INVALID_VALUE.
+ *   - int32: two's-complement wraparound (the exact SAT reduced mod 2^32), bit-exact and
+ *     deterministic.  fp32: IEEE adds in an unspecified, run-dependent association; every entry
+ *     satisfies |dst - exact| <= (rows+cols) * 1.2e-7 * SAT(|src|) at that entry (R10).
+ *   - libsat owns its workspace (per-tile aggregates, status words, tile counter), cached per
+ *     (device, stream) and grown on demand with cudaMalloc; growth is the only synchronising
+ *     event and must not happen inside CUDA-graph capture (call once before capturing).
+ */
+#ifndef LIBSAT_SAT_H
+#define LIBSAT_SAT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SAT_VERSION 100 /* 1.0.0 */
+
+typedef enum {
+    SAT_OK = 0,
+    SAT_ERR_INVALID_VALUE = 1,
+    SAT_ERR_MISALIGNED = 2,
+    SAT_ERR_UNSUPPORTED = 3,
+    SAT_ERR_OUT_OF_MEMORY = 4,
+    SAT_ERR_CUDA = 5,
+    SAT_ERR_NCCL = 6
+} sat_status_t;
+
+typedef enum { SAT_INT32 = 0, SAT_FLOAT32 = 1 } sat_dtype_t;
+
+/* Opaque multi-GPU communicator (owns an ncclComm_t).  Created by sat_comm_init, freed by
+ * sat_comm_destroy; owned by the caller. */
+typedef struct sat_comm_s* sat_comm_t;
+
+/* ------------------------------------------------------------------ single GPU (the hot path) */
+
+/* SAT of an int32 matrix, one pass, uint32 wraparound.
+ *   src   device, rows x cols, row stride `pitch` elements; read once.
+ *   dst   device, same shape and pitch; written once; may equal src.
+ * Errors: INVALID_VALUE (sizes, overlap), MISALIGNED, OUT_OF_MEMORY (workspace), CUDA (launch). */
+sat_status_t sat_compute_i32(const int32_t* src, int32_t* dst, int64_t rows, int64_t cols,
+                             int64_t pitch, void* stream);
+
+/* SAT of an fp32 matrix (the paper's "4-byte float"); tolerance rule above. */
+sat_status_t sat_compute_f32(const float* src, float* dst, int64_t rows, int64_t cols,
+                             int64_t pitch, void* stream);
+
+/* Same as above for either dtype, plus an optional carry row.
+ *   carry  device, `cols` elements of the same dtype, or NULL.  When given, carry[j] is added to
+ *          every element of column j of the result: dst[i][j] = carry[j] + SAT(src)[i][j].  With
+ *          carry = the last SAT row of the matrix above (a strip's "carry row", R12),
+ *          dst is that strip of the SAT of the stacked matrix. */
+sat_status_t sat_compute(sat_dtype_t dtype, const void* src, void* dst, int64_t rows, int64_t cols,
+                         int64_t pitch, const void* carry, void* stream);
+
+/* End-to-end call with HOST buffers: copies src host->device, computes the SAT, copies the result
+ * device->host and synchronises `stream` before returning.  The matrix is pipelined in horizontal
+ * strips (H2D of strip k+1, SAT of strip k and D2H of strip k-1 overlap; strip k uses the last SAT
+ * row of strip k-1 as its carry row).  host_src/host_dst: rows x cols, row stride `pitch`
+ * elements, may be the same buffer; pinned memory gives full PCIe bandwidth.  Device staging
+ * buffers are owned by libsat (cached per device).  Synchronous. */
+sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,
+                              int64_t cols, int64_t pitch, void* stream);
+
+/* ------------------------------------------------------------------ multi-GPU strip partition */
+
+/* Column sums of a strip (not in the paper; BASELINE.json north_star's strip carry):
+ *   colsum[j] = sum_i src[i][j], 0 <= i < rows.   src device (rows x cols, pitch); colsum device,
+ *   cols elements.  Deterministic (fixed summation order). */
+sat_status_t sat_strip_colsum(sat_dtype_t dtype, const void* src, void* colsum, int64_t rows,
+                              int64_t cols, int64_t pitch, void* stream);
+
+/* Carry row of rank `rank` from the gathered column sums of all ranks:
+ *   C[j] = sum_{g < rank} gathered[g*cols + j]   (ascending g: same association on every rank)
+ *   carry[j] = C[0] + ... + C[j]                  (row-wise prefix)
+ * gathered device (nranks x cols), carry device (cols).  rank 0 gets the zero vector. */
+sat_status_t sat_carry_prefix(sat_dtype_t dtype, const void* gathered, int nranks, int rank,
+                              int64_t cols, void* carry, void* stream);
+
+/* NCCL bootstrap.  Rank 0 calls sat_comm_get_unique_id and ships the 128 bytes to the other
+ * ranks (the Python binding broadcasts them over the torch process group); every rank then calls
+ * sat_comm_init collectively.  NCCL is loaded with dlopen("libnccl.so.2") at first use (the copy
+ * torch already loaded).  Errors: NCCL (load or NCCL call failure), UNSUPPORTED (built without
+ * nccl.h). */
+sat_status_t sat_comm_get_unique_id(unsigned char id[128]);
+sat_status_t sat_comm_init(sat_comm_t* comm, const unsigned char id[128], int nranks, int rank);
+sat_status_t sat_comm_destroy(sat_comm_t comm);
+
+/* Strip-partitioned SAT over `nranks` GPUs, one process per GPU, called collectively in the same
+ * order on every rank with equal `cols`.  Rank r passes ITS horizontal strip: global rows
+ * [row0_r, row0_r + strip_rows) with row0_r = sum of strip_rows of ranks < r (strips may differ in
+ * height).  Steps: sat_strip_colsum -> ncclAllGather of the colsum vectors -> sat_carry_prefix ->
+ * sat_compute with that carry.  strip_src/strip_dst device (this rank), may be equal. */
+sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, const void* strip_src,
+                                 void* strip_dst, int64_t strip_rows, int64_t cols, int64_t pitch,
+                                 void* stream);
+
+/* ------------------------------------------------------------------ introspection */
+
+typedef struct {
+    int32_t tile_rows;     /* TR: rows per tile */
+    int32_t tile_cols;     /* TC: columns per tile */
+    int32_t tma;           /* 1 = TMA path, 0 = generic load/store path */
+    int32_t ctas;          /* persistent CTAs launched */
+    int64_t tiles;         /* ceil(rows/TR) * ceil(cols/TC) */
+    int64_t aux_bytes;     /* bytes of per-tile aggregate slots for this shape */
+    int32_t variant;       /* kernel variant index */
+    int32_t order;         /* 0 = diagonal-major (Fig. 9), 1 = row-major */
+} sat_plan_t;
+
+/* Fill `plan` with what sat_compute would launch for this problem (no launch, no allocation). */
+sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t cols, int64_t pitch,
+                            const void* src, const void* dst, sat_plan_t* plan);
+
+/* Tuning knobs (process-wide; for sweeps and tests).  variant: -1 = automatic choice;
+ * order: 0 = diagonal-major (Fig. 9), 1 = row-major; ctas_per_sm: 0 = occupancy maximum.
+ * Returns INVALID_VALUE for an unknown variant. */
+sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm);
+int sat_num_variants(void);
+/* Cap the total number of persistent CTAs (0 = no cap).  A cap of 1 runs the whole matrix on one
+ * CTA: the forward-progress test of the tile-counter protocol. */
+sat_status_t sat_set_max_ctas(int max_ctas);
+/* Tile shape of variant v (TR, TC), or INVALID_VALUE. */
+sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* tile_cols);
+
+/* Test hook: run the kernel's serial-number -> tile mapping on the device for an R x C tile grid.
+ * out: device int32[2*R*C], out[2s] = I, out[2s+1] = J of serial s. */
+sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out, void* stream);
+
+/* Free every cached workspace and staging buffer (synchronises the devices that own them). */
+sat_status_t sat_release_workspaces(void);
+
+const char* sat_status_string(sat_status_t s);
+const char* sat_last_error_detail(void);
+int sat_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LIBSAT_SAT_H */

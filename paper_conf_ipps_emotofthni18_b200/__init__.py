@@ -1,0 +1,232 @@
+"""libsat Python binding: single-pass summed area tables on B200 (sm_100a).
+
+Thin marshalling over the C ABI of include/sat.h (same names).  Every step of the computation runs
+in libsat's CUDA kernels; PyTorch supplies device memory, streams and process groups only.  There
+is no CPU fallback: importing this package without a built libsat.so raises ImportError.
+
+    import paper_conf_ipps_emotofthni18_b200 as sat
+    b = sat.sat(a)                       # a: 2-D int32/float32 CUDA tensor (row stride = pitch)
+    sat.sat(a, out=a)                    # in place
+    sat.sat_host(np_array)               # host buffers -> host result (H2D + SAT + D2H pipeline)
+    comm = sat.Comm(group)               # NCCL communicator over a torch process group
+    sat.sat_sharded(strip, comm=comm)    # strip-partitioned SAT across ranks
+"""
+from __future__ import annotations
+
+import ctypes
+
+from . import _lib
+from ._lib import SAT_FLOAT32, SAT_INT32, SatError, SatPlan, check
+
+_lib.lib()  # load now: fail loudly at import if the native library is missing
+
+__all__ = [
+    "sat", "sat_host", "compute", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "release_workspaces",
+    "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
+]
+
+
+def _torch():
+    import torch
+
+    return torch
+
+
+def _dtype_code(t) -> int:
+    torch = _torch()
+    if t.dtype == torch.int32:
+        return SAT_INT32
+    if t.dtype == torch.float32:
+        return SAT_FLOAT32
+    raise TypeError(f"libsat supports int32 and float32, got {t.dtype}")
+
+
+def _stream_ptr(stream) -> int:
+    torch = _torch()
+    s = torch.cuda.current_stream() if stream is None else stream
+    return int(s.cuda_stream)
+
+
+def _matrix(t, name: str):
+    if not t.is_cuda or t.dim() != 2 or t.stride(1) != 1 or (t.shape[0] > 1 and t.stride(0) < t.shape[1]):
+        raise ValueError(f"{name}: need a 2-D CUDA tensor with unit column stride and row stride >= cols")
+    return t.shape[0], t.shape[1], (t.stride(0) if t.shape[0] > 1 else max(t.stride(0), t.shape[1]))
+
+
+def compute(dtype: int, src_ptr: int, dst_ptr: int, rows: int, cols: int, pitch: int, carry_ptr: int = 0,
+            stream_ptr: int = 0) -> None:
+    """Raw C-ABI call sat_compute (device pointers)."""
+    check(_lib.lib().sat_compute(dtype, src_ptr, dst_ptr, rows, cols, pitch, carry_ptr or None, stream_ptr or None),
+          "sat_compute")
+
+
+def sat(src, out=None, *, carry=None, stream=None):
+    """SAT of a 2-D int32/float32 CUDA tensor.  ``out`` may be ``src`` (in place) or a tensor of
+    the same shape and row stride; ``carry`` (1-D, cols) is added to every row of the result."""
+    torch = _torch()
+    rows, cols, pitch = _matrix(src, "src")
+    if out is None:
+        out = torch.empty_strided((rows, cols), (pitch, 1), dtype=src.dtype, device=src.device)
+    orows, ocols, opitch = _matrix(out, "out")
+    if (orows, ocols, opitch) != (rows, cols, pitch) or out.dtype != src.dtype or out.device != src.device:
+        raise ValueError("out must match src in shape, row stride, dtype and device")
+    cptr = 0
+    if carry is not None:
+        if carry.dtype != src.dtype or carry.numel() != cols or not carry.is_contiguous() or carry.device != src.device:
+            raise ValueError("carry must be a contiguous vector of `cols` elements of src's dtype and device")
+        cptr = carry.data_ptr()
+    with torch.cuda.device(src.device):
+        compute(_dtype_code(src), src.data_ptr(), out.data_ptr(), rows, cols, pitch, cptr, _stream_ptr(stream))
+    return out
+
+
+def sat_host(src, out=None, *, stream=None):
+    """End-to-end C-ABI call with host buffers (numpy int32/float32 2-D arrays, or CPU torch tensors).
+    Copies in, computes, copies out; synchronous.  Returns ``out``."""
+    import numpy as np
+
+    torch = _torch()
+    arr = src.numpy() if hasattr(src, "numpy") and not isinstance(src, np.ndarray) else src
+    if arr.ndim != 2 or arr.dtype not in (np.int32, np.float32) or arr.strides[1] != 4:
+        raise ValueError("src must be a 2-D int32/float32 host array with unit column stride")
+    if out is None:
+        out = np.empty_like(arr)
+    oarr = out.numpy() if hasattr(out, "numpy") and not isinstance(out, np.ndarray) else out
+    if oarr.shape != arr.shape or oarr.dtype != arr.dtype or oarr.strides != arr.strides:
+        raise ValueError("out must match src in shape, dtype and strides")
+    rows, cols = arr.shape
+    pitch = arr.strides[0] // 4 if rows > 1 else cols
+    code = SAT_INT32 if arr.dtype == np.int32 else SAT_FLOAT32
+    check(_lib.lib().sat_compute_host(code, arr.ctypes.data, oarr.ctypes.data, rows, cols, pitch,
+                                      _stream_ptr(stream) if torch.cuda.is_available() else None),
+          "sat_compute_host")
+    return out
+
+
+def strip_colsum(src, out=None, *, stream=None):
+    """Column sums of a strip (device), deterministic order."""
+    torch = _torch()
+    rows, cols, pitch = _matrix(src, "src")
+    if out is None:
+        out = torch.empty(cols, dtype=src.dtype, device=src.device)
+    with torch.cuda.device(src.device):
+        check(_lib.lib().sat_strip_colsum(_dtype_code(src), src.data_ptr(), out.data_ptr(), rows, cols, pitch,
+                                          _stream_ptr(stream)), "sat_strip_colsum")
+    return out
+
+
+def carry_prefix(gathered, rank: int, out=None, *, stream=None):
+    """Carry row of ``rank`` from the (nranks x cols) gathered column sums (device)."""
+    torch = _torch()
+    if gathered.dim() != 2 or not gathered.is_contiguous():
+        raise ValueError("gathered must be a contiguous (nranks, cols) tensor")
+    nranks, cols = gathered.shape
+    if out is None:
+        out = torch.empty(cols, dtype=gathered.dtype, device=gathered.device)
+    with torch.cuda.device(gathered.device):
+        check(_lib.lib().sat_carry_prefix(_dtype_code(gathered), gathered.data_ptr(), nranks, rank, cols,
+                                          out.data_ptr(), _stream_ptr(stream)), "sat_carry_prefix")
+    return out
+
+
+def strip_bounds(rows: int, world: int, rank: int) -> tuple[int, int]:
+    """Horizontal strip of ``rank`` when ``rows`` global rows are split over ``world`` ranks:
+    returns (row0, nrows).  Strips are ceil(rows/world) tall; the last ones may be shorter or empty."""
+    if world < 1 or not 0 <= rank < world or rows < 0:
+        raise ValueError("bad strip partition arguments")
+    h = -(-rows // world)
+    row0 = min(rank * h, rows)
+    return row0, min(h, rows - row0)
+
+
+class Comm:
+    """NCCL communicator for sat_sharded, bootstrapped over a torch process group: rank 0 creates the
+    128-byte NCCL id, the group broadcasts it, every rank calls sat_comm_init collectively."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+
+        torch = _torch()
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        buf = ctypes.create_string_buffer(128)
+        if self.rank == 0:
+            check(_lib.lib().sat_comm_get_unique_id(buf), "sat_comm_get_unique_id")
+        backend = dist.get_backend(group)
+        dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
+        t = torch.frombuffer(bytearray(buf.raw), dtype=torch.uint8).to(dev)
+        dist.broadcast(t, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+        raw = bytes(t.cpu().tolist())
+        self._h = ctypes.c_void_p()
+        check(_lib.lib().sat_comm_init(ctypes.byref(self._h), raw, self.world, self.rank), "sat_comm_init")
+
+    def close(self):
+        if self._h:
+            _lib.lib().sat_comm_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def sat_sharded(strip, out=None, *, comm: Comm, stream=None):
+    """Strip-partitioned SAT: this rank's horizontal strip in, this rank's strip of the global SAT out.
+    Collective over ``comm`` (call on every rank in the same order, equal column counts)."""
+    torch = _torch()
+    rows, cols, pitch = _matrix(strip, "strip") if strip.shape[0] > 0 else (0, strip.shape[1], strip.shape[1])
+    if out is None:
+        out = torch.empty_strided((rows, cols), (pitch, 1), dtype=strip.dtype, device=strip.device)
+    with torch.cuda.device(strip.device):
+        check(_lib.lib().sat_compute_sharded(comm._h, _dtype_code(strip), strip.data_ptr(), out.data_ptr(), rows,
+                                             cols, pitch, _stream_ptr(stream)), "sat_compute_sharded")
+    return out
+
+
+def query_plan(dtype: int, rows: int, cols: int, pitch: int | None = None, src_ptr: int = 0,
+               dst_ptr: int = 0) -> dict:
+    """What sat_compute would launch (tile shape, TMA or not, CTAs, tiles, aux bytes)."""
+    p = SatPlan()
+    check(_lib.lib().sat_query_plan(dtype, rows, cols, cols if pitch is None else pitch, src_ptr or None,
+                                    dst_ptr or None, ctypes.byref(p)), "sat_query_plan")
+    return {f: getattr(p, f) for f, _ in SatPlan._fields_}
+
+
+def set_tuning(variant: int = -1, order: int = 0, ctas_per_sm: int = 0) -> None:
+    check(_lib.lib().sat_set_tuning(variant, order, ctas_per_sm), "sat_set_tuning")
+
+
+def set_max_ctas(max_ctas: int = 0) -> None:
+    """Cap the persistent grid (0 = no cap); 1 = single-CTA forward-progress test."""
+    check(_lib.lib().sat_set_max_ctas(max_ctas), "sat_set_max_ctas")
+
+
+def num_variants() -> int:
+    return _lib.lib().sat_num_variants()
+
+
+def variant_info(v: int) -> tuple[int, int]:
+    tr, tc = ctypes.c_int32(), ctypes.c_int32()
+    check(_lib.lib().sat_variant_info(v, ctypes.byref(tr), ctypes.byref(tc)), "sat_variant_info")
+    return tr.value, tc.value
+
+
+def debug_tile_order(R: int, C: int, order: int = 0, device=None):
+    """The kernel's serial -> (I, J) map evaluated on the GPU: int32 tensor (R*C, 2)."""
+    torch = _torch()
+    out = torch.empty((R * C, 2), dtype=torch.int32, device=device or "cuda")
+    with torch.cuda.device(out.device):
+        check(_lib.lib().sat_debug_tile_order(R, C, order, out.data_ptr(), _stream_ptr(None)), "sat_debug_tile_order")
+    return out
+
+
+def release_workspaces() -> None:
+    check(_lib.lib().sat_release_workspaces(), "sat_release_workspaces")
+
+
+def version() -> int:
+    return _lib.lib().sat_version()

@@ -1,0 +1,817 @@
+// sat_api.cu -- libsat host side: the C ABI of include/sat.h.  Argument validation, the cached
+// per-(device, stream) workspace, TMA tensor maps, kernel variant selection and launch, the
+// end-to-end host-buffer pipeline and the NCCL strip-partitioned path.
+#include <dlfcn.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include <cudaTypedefs.h>  // PFN_cuTensorMapEncodeTiled
+
+#include "sat.h"
+#include "sat_aux_kernels.cuh"
+#include "sat_kernel.cuh"
+
+#if defined(SAT_HAVE_NCCL_H)
+#include <nccl.h>
+#endif
+
+#define SAT_API extern "C" __attribute__((visibility("default")))
+
+namespace {
+
+using sat::Ctrl;
+using sat::KParams;
+
+// ------------------------------------------------------------------ error reporting
+thread_local std::string g_detail;
+
+sat_status_t fail(sat_status_t s, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    g_detail = buf;
+    return s;
+}
+
+sat_status_t cuda_fail(cudaError_t e, const char* what) {
+    return fail(SAT_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+#define SAT_CUDA(call)                                  \
+    do {                                                \
+        cudaError_t e_ = (call);                        \
+        if (e_ != cudaSuccess) return cuda_fail(e_, #call); \
+    } while (0)
+
+// ------------------------------------------------------------------ kernel variants
+using LaunchFn = cudaError_t (*)(bool tma, bool carry, dim3 grid, cudaStream_t st, const CUtensorMap& mi,
+                                 const CUtensorMap& mo, const void* params);
+using PrepareFn = cudaError_t (*)(bool tma, bool carry, int* occupancy);
+
+struct Variant {
+    int TR, TC, NW, STAGES;
+    size_t smem;           // dynamic shared memory bytes (same for int32 / fp32)
+    LaunchFn launch[2];    // [dtype]
+    PrepareFn prepare[2];  // [dtype]
+};
+
+template <typename V, typename Cfg, bool TMA, bool CARRY>
+void* kernel_ptr() {
+    return reinterpret_cast<void*>(&sat::sat_tiles_kernel<V, Cfg, TMA, CARRY>);
+}
+
+template <typename V, typename Cfg>
+cudaError_t launch_variant(bool tma, bool carry, dim3 grid, cudaStream_t st, const CUtensorMap& mi,
+                           const CUtensorMap& mo, const void* params) {
+    const KParams<V>& p = *static_cast<const KParams<V>*>(params);
+    const size_t smem = sizeof(sat::Smem<V, Cfg>);
+    const dim3 block(Cfg::NW * 32);
+    if (tma) {
+        if (carry) sat::sat_tiles_kernel<V, Cfg, true, true><<<grid, block, smem, st>>>(mi, mo, p);
+        else sat::sat_tiles_kernel<V, Cfg, true, false><<<grid, block, smem, st>>>(mi, mo, p);
+    } else {
+        if (carry) sat::sat_tiles_kernel<V, Cfg, false, true><<<grid, block, smem, st>>>(mi, mo, p);
+        else sat::sat_tiles_kernel<V, Cfg, false, false><<<grid, block, smem, st>>>(mi, mo, p);
+    }
+    return cudaGetLastError();
+}
+
+template <typename V, typename Cfg>
+cudaError_t prepare_variant(bool tma, bool carry, int* occupancy) {
+    void* k = tma ? (carry ? kernel_ptr<V, Cfg, true, true>() : kernel_ptr<V, Cfg, true, false>())
+                  : (carry ? kernel_ptr<V, Cfg, false, true>() : kernel_ptr<V, Cfg, false, false>());
+    const int smem = static_cast<int>(sizeof(sat::Smem<V, Cfg>));
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy, k, Cfg::NW * 32, smem);
+}
+
+template <typename Cfg>
+Variant make_variant() {
+    Variant v;
+    v.TR = Cfg::TR;
+    v.TC = Cfg::TC;
+    v.NW = Cfg::NW;
+    v.STAGES = Cfg::STAGES;
+    v.smem = sizeof(sat::Smem<uint32_t, Cfg>);
+    v.launch[SAT_INT32] = &launch_variant<uint32_t, Cfg>;
+    v.launch[SAT_FLOAT32] = &launch_variant<float, Cfg>;
+    v.prepare[SAT_INT32] = &prepare_variant<uint32_t, Cfg>;
+    v.prepare[SAT_FLOAT32] = &prepare_variant<float, Cfg>;
+    return v;
+}
+
+const std::vector<Variant>& variants() {
+    static const std::vector<Variant> vs = {
+        make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 0: 32 KiB tiles, 2 stages
+        make_variant<sat::TileCfg<64, 128, 8, 3>>(),   // 1: 32 KiB tiles, 3 stages
+        make_variant<sat::TileCfg<32, 128, 8, 3>>(),   // 2: 16 KiB tiles, 3 stages
+        make_variant<sat::TileCfg<128, 128, 8, 2>>(),  // 3: 64 KiB tiles (the paper's W=128), 2 stages
+        make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 4: 64 KiB tiles, 512 threads
+        make_variant<sat::TileCfg<32, 128, 8, 4>>(),   // 5: 16 KiB tiles, 4 stages
+    };
+    return vs;
+}
+
+// process-wide tuning knobs (sat_set_tuning)
+std::mutex g_mu;
+int g_variant = -1;
+int g_order = 0;
+int g_ctas_per_sm = 0;
+int g_max_ctas = 0;
+
+int auto_variant(int64_t rows, int64_t cols) {
+    (void)cols;
+    (void)rows;
+    return 0;
+}
+
+// ------------------------------------------------------------------ device info caches
+struct DeviceInfo {
+    int sms = 0;
+    std::map<std::pair<int, int>, int> occ;  // (variant*8 + dtype*4 + tma*2 + carry) -> occupancy
+};
+std::map<int, DeviceInfo> g_dev;
+
+sat_status_t device_info(int dev, DeviceInfo** out) {
+    auto it = g_dev.find(dev);
+    if (it == g_dev.end()) {
+        DeviceInfo di;
+        SAT_CUDA(cudaDeviceGetAttribute(&di.sms, cudaDevAttrMultiProcessorCount, dev));
+        it = g_dev.emplace(dev, di).first;
+    }
+    *out = &it->second;
+    return SAT_OK;
+}
+
+sat_status_t occupancy(int dev, int vi, sat_dtype_t dt, bool tma, bool carry, int* occ) {
+    DeviceInfo* di;
+    sat_status_t s = device_info(dev, &di);
+    if (s != SAT_OK) return s;
+    const std::pair<int, int> key(vi, dt * 4 + (tma ? 2 : 0) + (carry ? 1 : 0));
+    auto it = di->occ.find(key);
+    if (it == di->occ.end()) {
+        int o = 0;
+        cudaError_t e = variants()[vi].prepare[dt](tma, carry, &o);
+        if (e != cudaSuccess) return cuda_fail(e, "kernel attribute / occupancy query");
+        if (o < 1) return fail(SAT_ERR_UNSUPPORTED, "kernel variant %d does not fit on an SM", vi);
+        it = di->occ.emplace(key, o).first;
+    }
+    *occ = it->second;
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ workspace
+struct Workspace {
+    int dev = 0;
+    cudaStream_t stream = nullptr;
+    Ctrl* ctrl = nullptr;
+    uint64_t* slots = nullptr;
+    size_t slot_words = 0;
+    uint64_t calls = 0;
+    void* scratch = nullptr;  // colsum partials etc.
+    size_t scratch_bytes = 0;
+};
+std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
+
+sat_status_t reset_ctrl(Workspace* w) {
+    Ctrl init{0u, 0u, 1u, 0u};
+    SAT_CUDA(cudaMemcpyAsync(w->ctrl, &init, sizeof(Ctrl), cudaMemcpyHostToDevice, w->stream));
+    SAT_CUDA(cudaStreamSynchronize(w->stream));
+    return SAT_OK;
+}
+
+sat_status_t get_workspace(int dev, cudaStream_t st, size_t slot_words, Workspace** out) {
+    auto key = std::make_pair(dev, st);
+    auto it = g_ws.find(key);
+    Workspace* w;
+    if (it == g_ws.end()) {
+        w = new Workspace();
+        w->dev = dev;
+        w->stream = st;
+        cudaError_t e = cudaMalloc(&w->ctrl, 256);
+        if (e != cudaSuccess) {
+            delete w;
+            return fail(SAT_ERR_OUT_OF_MEMORY, "workspace control block: %s", cudaGetErrorString(e));
+        }
+        sat_status_t s = reset_ctrl(w);
+        if (s != SAT_OK) {
+            cudaFree(w->ctrl);
+            delete w;
+            return s;
+        }
+        g_ws[key] = w;
+    } else {
+        w = it->second;
+    }
+    if (slot_words > w->slot_words) {
+        size_t want = slot_words + slot_words / 4;
+        SAT_CUDA(cudaStreamSynchronize(st));
+        if (w->slots) SAT_CUDA(cudaFree(w->slots));
+        w->slots = nullptr;
+        w->slot_words = 0;
+        cudaError_t e = cudaMalloc(&w->slots, want * sizeof(uint64_t));
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(SAT_ERR_OUT_OF_MEMORY, "workspace slots (%zu bytes): %s", want * 8, cudaGetErrorString(e));
+        }
+        SAT_CUDA(cudaMemsetAsync(w->slots, 0, want * sizeof(uint64_t), st));
+        w->slot_words = want;
+    }
+    // Epoch wrap (after ~2^30 launches on this workspace): clear the slots and restart at epoch 1.
+    if (w->calls + 2 >= sat::kEpochMax) {
+        SAT_CUDA(cudaStreamSynchronize(st));
+        SAT_CUDA(cudaMemsetAsync(w->slots, 0, w->slot_words * sizeof(uint64_t), st));
+        sat_status_t s = reset_ctrl(w);
+        if (s != SAT_OK) return s;
+        w->calls = 0;
+    }
+    *out = w;
+    return SAT_OK;
+}
+
+sat_status_t get_scratch(Workspace* w, size_t bytes, void** out) {
+    if (bytes > w->scratch_bytes) {
+        SAT_CUDA(cudaStreamSynchronize(w->stream));
+        if (w->scratch) SAT_CUDA(cudaFree(w->scratch));
+        w->scratch = nullptr;
+        w->scratch_bytes = 0;
+        cudaError_t e = cudaMalloc(&w->scratch, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(SAT_ERR_OUT_OF_MEMORY, "scratch (%zu bytes): %s", bytes, cudaGetErrorString(e));
+        }
+        w->scratch_bytes = bytes;
+    }
+    *out = w->scratch;
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ TMA tensor maps
+PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
+
+sat_status_t get_encoder() {
+    if (g_encode) return SAT_OK;
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !fn)
+        return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled entry point unavailable (%s)", cudaGetErrorString(e));
+    g_encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+    return SAT_OK;
+}
+
+sat_status_t encode_map(CUtensorMap* m, sat_dtype_t dt, const void* ptr, int64_t rows, int64_t cols, int64_t pitch,
+                        int TR, int TC) {
+    cuuint64_t dims[2] = {static_cast<cuuint64_t>(cols), static_cast<cuuint64_t>(rows)};
+    cuuint64_t strides[1] = {static_cast<cuuint64_t>(pitch) * 4u};
+    cuuint32_t box[2] = {static_cast<cuuint32_t>(TC), static_cast<cuuint32_t>(TR)};
+    cuuint32_t estr[2] = {1u, 1u};
+    CUresult r = g_encode(m, dt == SAT_FLOAT32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_UINT32, 2,
+                          const_cast<void*>(ptr), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                          CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled failed (CUresult %d)", (int)r);
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ validation / planning
+sat_status_t validate(const void* src, const void* dst, int64_t rows, int64_t cols, int64_t pitch) {
+    if (rows < 0 || cols < 0 || pitch < cols)
+        return fail(SAT_ERR_INVALID_VALUE, "bad sizes rows=%lld cols=%lld pitch=%lld", (long long)rows,
+                    (long long)cols, (long long)pitch);
+    if (rows == 0 || cols == 0) return SAT_OK;
+    if (!src || !dst) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 3u)
+        return fail(SAT_ERR_MISALIGNED, "pointers must be 4-byte aligned");
+    if (src != dst) {
+        const uintptr_t bytes = static_cast<uintptr_t>(((rows - 1) * pitch + cols) * 4);
+        const uintptr_t a = reinterpret_cast<uintptr_t>(src), b = reinterpret_cast<uintptr_t>(dst);
+        if (a < b + bytes && b < a + bytes) return fail(SAT_ERR_INVALID_VALUE, "src and dst partially overlap");
+    }
+    if (rows > (int64_t(1) << 31) - 1 || cols > (int64_t(1) << 31) - 1)
+        return fail(SAT_ERR_UNSUPPORTED, "rows and cols must be < 2^31");
+    return SAT_OK;
+}
+
+bool tma_ok(const void* src, const void* dst, int64_t pitch) {
+    return ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15u) == 0 &&
+           ((pitch * 4) % 16) == 0 && pitch * 4 < (int64_t(1) << 40);
+}
+
+struct Plan {
+    int vi, TR, TC, R, C, order;
+    int64_t ntiles;
+    bool tma;
+};
+
+sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* src, const void* dst, Plan* pl) {
+    int vi, order;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        vi = g_variant >= 0 ? g_variant : auto_variant(rows, cols);
+        order = g_order;
+    }
+    const Variant& v = variants()[vi];
+    pl->vi = vi;
+    pl->TR = v.TR;
+    pl->TC = v.TC;
+    pl->R = static_cast<int>((rows + v.TR - 1) / v.TR);
+    pl->C = static_cast<int>((cols + v.TC - 1) / v.TC);
+    pl->ntiles = static_cast<int64_t>(pl->R) * pl->C;
+    pl->order = order;
+    pl->tma = tma_ok(src, dst, pitch);
+    if (pl->ntiles > (int64_t(1) << 31) - 4096)
+        return fail(SAT_ERR_UNSUPPORTED, "too many tiles (%lld)", (long long)pl->ntiles);
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ the hot path
+sat_status_t compute_impl(sat_dtype_t dt, const void* src, void* dst, int64_t rows, int64_t cols, int64_t pitch,
+                          const void* carry, cudaStream_t st) {
+    if (dt != SAT_INT32 && dt != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dt);
+    sat_status_t s = validate(src, dst, rows, cols, pitch);
+    if (s != SAT_OK || rows == 0 || cols == 0) return s;
+    if (carry && (reinterpret_cast<uintptr_t>(carry) & 3u)) return fail(SAT_ERR_MISALIGNED, "carry misaligned");
+    Plan pl;
+    if ((s = make_plan(rows, cols, pitch, src, dst, &pl)) != SAT_OK) return s;
+    const Variant& v = variants()[pl.vi];
+
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    int occ = 0;
+    if ((s = occupancy(dev, pl.vi, dt, pl.tma, carry != nullptr, &occ)) != SAT_OK) return s;
+    DeviceInfo* di;
+    if ((s = device_info(dev, &di)) != SAT_OK) return s;
+    int per_sm = (g_ctas_per_sm > 0 && g_ctas_per_sm < occ) ? g_ctas_per_sm : occ;
+    int64_t grid = static_cast<int64_t>(di->sms) * per_sm;
+    if (g_max_ctas > 0 && grid > g_max_ctas) grid = g_max_ctas;
+    if (grid > pl.ntiles) grid = pl.ntiles;
+
+    Workspace* w;
+    const size_t words = static_cast<size_t>(pl.ntiles) * (v.TR + v.TC + 1);
+    if ((s = get_workspace(dev, st, words, &w)) != SAT_OK) return s;
+
+    CUtensorMap mi, mo;
+    std::memset(&mi, 0, sizeof(mi));
+    std::memset(&mo, 0, sizeof(mo));
+    if (pl.tma) {
+        if ((s = get_encoder()) != SAT_OK) return s;
+        if ((s = encode_map(&mi, dt, src, rows, cols, pitch, v.TR, v.TC)) != SAT_OK) return s;
+        if ((s = encode_map(&mo, dt, dst, rows, cols, pitch, v.TR, v.TC)) != SAT_OK) return s;
+    }
+    KParams<uint32_t> p;  // identical layout for float
+    p.src = static_cast<const uint32_t*>(src);
+    p.dst = static_cast<uint32_t*>(dst);
+    p.rows = rows;
+    p.cols = cols;
+    p.pitch = pitch;
+    p.R = pl.R;
+    p.C = pl.C;
+    p.ntiles = static_cast<int>(pl.ntiles);
+    p.order = pl.order;
+    p.row_slots = w->slots;
+    p.col_slots = w->slots + static_cast<size_t>(pl.ntiles) * v.TR;
+    p.corner_slots = w->slots + static_cast<size_t>(pl.ntiles) * (v.TR + v.TC);
+    p.ctrl = w->ctrl;
+    p.carry = static_cast<const uint32_t*>(carry);
+    cudaError_t e = v.launch[dt](pl.tma, carry != nullptr, dim3(static_cast<unsigned>(grid)), st, mi, mo, &p);
+    if (e != cudaSuccess) return cuda_fail(e, "sat_tiles_kernel launch");
+    w->calls++;
+    return SAT_OK;
+}
+
+sat_status_t colsum_impl(sat_dtype_t dt, const void* src, void* colsum, int64_t rows, int64_t cols, int64_t pitch,
+                         cudaStream_t st) {
+    if (dt != SAT_INT32 && dt != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dt);
+    if (rows < 0 || cols < 0 || pitch < cols) return fail(SAT_ERR_INVALID_VALUE, "bad sizes");
+    if (cols == 0) return SAT_OK;
+    if (!colsum || (rows > 0 && !src)) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    if ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(colsum)) & 3u)
+        return fail(SAT_ERR_MISALIGNED, "pointers must be 4-byte aligned");
+    if (rows == 0) {
+        SAT_CUDA(cudaMemsetAsync(colsum, 0, cols * 4, st));
+        return SAT_OK;
+    }
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    DeviceInfo* di;
+    sat_status_t s = device_info(dev, &di);
+    if (s != SAT_OK) return s;
+    const int64_t bx = (cols + 255) / 256;
+    int64_t nseg = (static_cast<int64_t>(di->sms) * 8 + bx - 1) / bx;
+    const int64_t max_seg = (rows + 7) / 8;
+    if (nseg > max_seg) nseg = max_seg;
+    if (nseg > 65535) nseg = 65535;
+    if (nseg < 1) nseg = 1;
+    const int64_t seg = (rows + nseg - 1) / nseg;
+    nseg = (rows + seg - 1) / seg;
+    Workspace* w;
+    if ((s = get_workspace(dev, st, 0, &w)) != SAT_OK) return s;
+    void* partial;
+    if ((s = get_scratch(w, static_cast<size_t>(nseg * cols) * 4, &partial)) != SAT_OK) return s;
+    dim3 g1(static_cast<unsigned>(bx), static_cast<unsigned>(nseg));
+    if (dt == SAT_INT32) {
+        sat::colsum_partial_kernel<uint32_t><<<g1, 256, 0, st>>>(static_cast<const uint32_t*>(src),
+                                                                 static_cast<uint32_t*>(partial), rows, cols, pitch, seg);
+        sat::colsum_reduce_kernel<uint32_t><<<static_cast<unsigned>((cols + 255) / 256), 256, 0, st>>>(
+            static_cast<const uint32_t*>(partial), static_cast<uint32_t*>(colsum), cols, static_cast<int>(nseg));
+    } else {
+        sat::colsum_partial_kernel<float><<<g1, 256, 0, st>>>(static_cast<const float*>(src),
+                                                              static_cast<float*>(partial), rows, cols, pitch, seg);
+        sat::colsum_reduce_kernel<float><<<static_cast<unsigned>((cols + 255) / 256), 256, 0, st>>>(
+            static_cast<const float*>(partial), static_cast<float*>(colsum), cols, static_cast<int>(nseg));
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "colsum kernels");
+    return SAT_OK;
+}
+
+sat_status_t carry_impl(sat_dtype_t dt, const void* gathered, int nranks, int rank, int64_t cols, void* carry,
+                        cudaStream_t st) {
+    if (dt != SAT_INT32 && dt != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dt);
+    if (nranks < 1 || rank < 0 || rank >= nranks || cols < 0) return fail(SAT_ERR_INVALID_VALUE, "bad rank/sizes");
+    if (cols == 0) return SAT_OK;
+    if (!carry || (rank > 0 && !gathered)) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    if (dt == SAT_INT32)
+        sat::carry_prefix_kernel<uint32_t><<<1, 1024, 0, st>>>(static_cast<const uint32_t*>(gathered), rank, cols,
+                                                               static_cast<uint32_t*>(carry));
+    else
+        sat::carry_prefix_kernel<float><<<1, 1024, 0, st>>>(static_cast<const float*>(gathered), rank, cols,
+                                                            static_cast<float*>(carry));
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "carry_prefix_kernel");
+    return SAT_OK;
+}
+
+// ------------------------------------------------------------------ end-to-end host pipeline
+struct Staging {
+    void* buf = nullptr;
+    size_t bytes = 0;
+    cudaStream_t h2d = nullptr, d2h = nullptr;
+};
+std::map<int, Staging> g_staging;
+
+// ------------------------------------------------------------------ NCCL (dlopen)
+#if defined(SAT_HAVE_NCCL_H)
+struct NcclApi {
+    void* h = nullptr;
+    ncclResult_t (*getUniqueId)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*commInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*commDestroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*allGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+    const char* (*errStr)(ncclResult_t) = nullptr;
+};
+NcclApi g_nccl;
+
+sat_status_t load_nccl() {
+    if (g_nccl.h) return SAT_OK;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return fail(SAT_ERR_NCCL, "dlopen(libnccl.so.2) failed: %s", dlerror());
+    g_nccl.getUniqueId = reinterpret_cast<decltype(g_nccl.getUniqueId)>(dlsym(h, "ncclGetUniqueId"));
+    g_nccl.commInitRank = reinterpret_cast<decltype(g_nccl.commInitRank)>(dlsym(h, "ncclCommInitRank"));
+    g_nccl.commDestroy = reinterpret_cast<decltype(g_nccl.commDestroy)>(dlsym(h, "ncclCommDestroy"));
+    g_nccl.allGather = reinterpret_cast<decltype(g_nccl.allGather)>(dlsym(h, "ncclAllGather"));
+    g_nccl.errStr = reinterpret_cast<decltype(g_nccl.errStr)>(dlsym(h, "ncclGetErrorString"));
+    if (!g_nccl.getUniqueId || !g_nccl.commInitRank || !g_nccl.commDestroy || !g_nccl.allGather || !g_nccl.errStr)
+        return fail(SAT_ERR_NCCL, "libnccl.so.2 lacks a required symbol");
+    g_nccl.h = h;
+    return SAT_OK;
+}
+
+sat_status_t nccl_fail(ncclResult_t r, const char* what) {
+    return fail(SAT_ERR_NCCL, "%s: %s", what, g_nccl.errStr ? g_nccl.errStr(r) : "?");
+}
+#endif
+
+}  // namespace
+
+struct sat_comm_s {
+#if defined(SAT_HAVE_NCCL_H)
+    ncclComm_t comm = nullptr;
+#endif
+    int nranks = 0, rank = 0, dev = 0;
+    void* buf = nullptr;  // colsum [cols] | gathered [nranks*cols] | carry [cols]
+    size_t bytes = 0;
+};
+
+// ====================================================================== C ABI
+SAT_API sat_status_t sat_compute(sat_dtype_t dtype, const void* src, void* dst, int64_t rows, int64_t cols,
+                                 int64_t pitch, const void* carry, void* stream) {
+    return compute_impl(dtype, src, dst, rows, cols, pitch, carry, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_compute_i32(const int32_t* src, int32_t* dst, int64_t rows, int64_t cols, int64_t pitch,
+                                     void* stream) {
+    return compute_impl(SAT_INT32, src, dst, rows, cols, pitch, nullptr, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_compute_f32(const float* src, float* dst, int64_t rows, int64_t cols, int64_t pitch,
+                                     void* stream) {
+    return compute_impl(SAT_FLOAT32, src, dst, rows, cols, pitch, nullptr, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_strip_colsum(sat_dtype_t dtype, const void* src, void* colsum, int64_t rows, int64_t cols,
+                                      int64_t pitch, void* stream) {
+    return colsum_impl(dtype, src, colsum, rows, cols, pitch, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_carry_prefix(sat_dtype_t dtype, const void* gathered, int nranks, int rank, int64_t cols,
+                                      void* carry, void* stream) {
+    return carry_impl(dtype, gathered, nranks, rank, cols, carry, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,
+                                      int64_t cols, int64_t pitch, void* stream) {
+    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype");
+    if (rows < 0 || cols < 0 || pitch < cols) return fail(SAT_ERR_INVALID_VALUE, "bad sizes");
+    if (rows == 0 || cols == 0) return SAT_OK;
+    if (!host_src || !host_dst) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    Staging* sg;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        sg = &g_staging[dev];
+        const size_t bytes = static_cast<size_t>(rows) * pitch * 4;
+        if (!sg->h2d) {
+            SAT_CUDA(cudaStreamCreateWithFlags(&sg->h2d, cudaStreamNonBlocking));
+            SAT_CUDA(cudaStreamCreateWithFlags(&sg->d2h, cudaStreamNonBlocking));
+        }
+        if (bytes > sg->bytes) {
+            if (sg->buf) SAT_CUDA(cudaFree(sg->buf));
+            sg->buf = nullptr;
+            sg->bytes = 0;
+            cudaError_t e = cudaMalloc(&sg->buf, bytes);
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                return fail(SAT_ERR_OUT_OF_MEMORY, "staging buffer (%zu bytes)", bytes);
+            }
+            sg->bytes = bytes;
+        }
+    }
+    // strips of >= 2 MiB, at most 16, multiples of 128 rows
+    const int64_t row_bytes = pitch * 4;
+    int64_t nstrips = (rows * row_bytes) / (int64_t(2) << 20);
+    if (nstrips < 1) nstrips = 1;
+    if (nstrips > 16) nstrips = 16;
+    int64_t h = (rows + nstrips - 1) / nstrips;
+    h = ((h + 127) / 128) * 128;
+    nstrips = (rows + h - 1) / h;
+    std::vector<cudaEvent_t> ev(2 * nstrips);
+    for (auto& e : ev) SAT_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    sat_status_t status = SAT_OK;
+    char* dbuf = static_cast<char*>(sg->buf);
+    for (int64_t k = 0; k < nstrips && status == SAT_OK; ++k) {
+        const int64_t r0 = k * h;
+        const int64_t nr = (r0 + h <= rows) ? h : rows - r0;
+        char* dstrip = dbuf + r0 * row_bytes;
+        const char* hs = static_cast<const char*>(host_src) + r0 * row_bytes;
+        char* hd = static_cast<char*>(host_dst) + r0 * row_bytes;
+        cudaError_t e = cudaMemcpy2DAsync(dstrip, row_bytes, hs, row_bytes, cols * 4, nr, cudaMemcpyHostToDevice,
+                                          sg->h2d);
+        if (e == cudaSuccess) e = cudaEventRecord(ev[2 * k], sg->h2d);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(st, ev[2 * k], 0);
+        if (e != cudaSuccess) {
+            status = cuda_fail(e, "host pipeline H2D");
+            break;
+        }
+        const void* carry = (k > 0) ? static_cast<const void*>(dstrip - row_bytes) : nullptr;
+        status = compute_impl(dtype, dstrip, dstrip, nr, cols, pitch, carry, st);
+        if (status != SAT_OK) break;
+        e = cudaEventRecord(ev[2 * k + 1], st);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(sg->d2h, ev[2 * k + 1], 0);
+        if (e == cudaSuccess)
+            e = cudaMemcpy2DAsync(hd, row_bytes, dstrip, row_bytes, cols * 4, nr, cudaMemcpyDeviceToHost, sg->d2h);
+        if (e != cudaSuccess) status = cuda_fail(e, "host pipeline D2H");
+    }
+    cudaError_t e1 = cudaStreamSynchronize(sg->d2h);
+    cudaError_t e2 = cudaStreamSynchronize(st);
+    cudaError_t e3 = cudaStreamSynchronize(sg->h2d);
+    for (auto& e : ev) cudaEventDestroy(e);
+    if (status != SAT_OK) return status;
+    if (e1 != cudaSuccess) return cuda_fail(e1, "host pipeline sync");
+    if (e2 != cudaSuccess) return cuda_fail(e2, "host pipeline sync");
+    if (e3 != cudaSuccess) return cuda_fail(e3, "host pipeline sync");
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_comm_get_unique_id(unsigned char id[128]) {
+#if defined(SAT_HAVE_NCCL_H)
+    if (!id) return fail(SAT_ERR_INVALID_VALUE, "null id");
+    sat_status_t s = load_nccl();
+    if (s != SAT_OK) return s;
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    ncclUniqueId uid;
+    ncclResult_t r = g_nccl.getUniqueId(&uid);
+    if (r != ncclSuccess) return nccl_fail(r, "ncclGetUniqueId");
+    std::memcpy(id, &uid, 128);
+    return SAT_OK;
+#else
+    (void)id;
+    return fail(SAT_ERR_UNSUPPORTED, "libsat was built without nccl.h");
+#endif
+}
+
+SAT_API sat_status_t sat_comm_init(sat_comm_t* comm, const unsigned char id[128], int nranks, int rank) {
+#if defined(SAT_HAVE_NCCL_H)
+    if (!comm || !id || nranks < 1 || rank < 0 || rank >= nranks) return fail(SAT_ERR_INVALID_VALUE, "bad args");
+    sat_status_t s = load_nccl();
+    if (s != SAT_OK) return s;
+    auto* c = new sat_comm_s();
+    c->nranks = nranks;
+    c->rank = rank;
+    cudaGetDevice(&c->dev);
+    ncclUniqueId uid;
+    std::memcpy(&uid, id, 128);
+    ncclResult_t r = g_nccl.commInitRank(&c->comm, nranks, uid, rank);
+    if (r != ncclSuccess) {
+        delete c;
+        return nccl_fail(r, "ncclCommInitRank");
+    }
+    *comm = c;
+    return SAT_OK;
+#else
+    (void)comm; (void)id; (void)nranks; (void)rank;
+    return fail(SAT_ERR_UNSUPPORTED, "libsat was built without nccl.h");
+#endif
+}
+
+SAT_API sat_status_t sat_comm_destroy(sat_comm_t comm) {
+    if (!comm) return SAT_OK;
+#if defined(SAT_HAVE_NCCL_H)
+    if (comm->comm) g_nccl.commDestroy(comm->comm);
+#endif
+    if (comm->buf) cudaFree(comm->buf);
+    delete comm;
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, const void* strip_src, void* strip_dst,
+                                         int64_t strip_rows, int64_t cols, int64_t pitch, void* stream) {
+#if defined(SAT_HAVE_NCCL_H)
+    if (!comm) return fail(SAT_ERR_INVALID_VALUE, "null comm");
+    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype");
+    if (strip_rows < 0 || cols <= 0 || pitch < cols) return fail(SAT_ERR_INVALID_VALUE, "bad sizes");
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const size_t need = static_cast<size_t>(cols) * 4 * (comm->nranks + 2);
+    if (need > comm->bytes) {
+        if (comm->buf) SAT_CUDA(cudaFree(comm->buf));
+        comm->buf = nullptr;
+        comm->bytes = 0;
+        cudaError_t e = cudaMalloc(&comm->buf, need);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(SAT_ERR_OUT_OF_MEMORY, "sharded buffers");
+        }
+        comm->bytes = need;
+    }
+    char* base = static_cast<char*>(comm->buf);
+    void* colsum = base;
+    void* gathered = base + cols * 4;
+    void* carry = base + cols * 4 * (comm->nranks + 1);
+    sat_status_t s = colsum_impl(dtype, strip_src, colsum, strip_rows, cols, pitch, st);
+    if (s != SAT_OK) return s;
+    ncclResult_t r = g_nccl.allGather(colsum, gathered, static_cast<size_t>(cols),
+                                      dtype == SAT_INT32 ? ncclUint32 : ncclFloat32, comm->comm, st);
+    if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
+    if ((s = carry_impl(dtype, gathered, comm->nranks, comm->rank, cols, carry, st)) != SAT_OK) return s;
+    if (strip_rows == 0) return SAT_OK;
+    return compute_impl(dtype, strip_src, strip_dst, strip_rows, cols, pitch, carry, st);
+#else
+    (void)comm; (void)dtype; (void)strip_src; (void)strip_dst; (void)strip_rows; (void)cols; (void)pitch; (void)stream;
+    return fail(SAT_ERR_UNSUPPORTED, "libsat was built without nccl.h");
+#endif
+}
+
+SAT_API sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t cols, int64_t pitch, const void* src,
+                                    const void* dst, sat_plan_t* plan) {
+    if (!plan) return fail(SAT_ERR_INVALID_VALUE, "null plan");
+    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype");
+    if (rows <= 0 || cols <= 0 || pitch < cols) return fail(SAT_ERR_INVALID_VALUE, "bad sizes");
+    Plan pl;
+    sat_status_t s = make_plan(rows, cols, pitch, src, dst, &pl);
+    if (s != SAT_OK) return s;
+    const Variant& v = variants()[pl.vi];
+    plan->tile_rows = v.TR;
+    plan->tile_cols = v.TC;
+    plan->tma = pl.tma ? 1 : 0;
+    plan->tiles = pl.ntiles;
+    plan->aux_bytes = pl.ntiles * (v.TR + v.TC + 1) * 8;
+    plan->variant = pl.vi;
+    plan->order = pl.order;
+    plan->ctas = 0;
+    int dev = 0;
+    if (cudaGetDevice(&dev) == cudaSuccess) {
+        std::lock_guard<std::mutex> lk(g_mu);
+        int occ = 0;
+        DeviceInfo* di;
+        if (occupancy(dev, pl.vi, dtype, pl.tma, false, &occ) == SAT_OK && device_info(dev, &di) == SAT_OK) {
+            int per_sm = (g_ctas_per_sm > 0 && g_ctas_per_sm < occ) ? g_ctas_per_sm : occ;
+            int64_t grid = static_cast<int64_t>(di->sms) * per_sm;
+            if (g_max_ctas > 0 && grid > g_max_ctas) grid = g_max_ctas;
+            plan->ctas = static_cast<int32_t>(grid < pl.ntiles ? grid : pl.ntiles);
+        }
+    }
+    cudaGetLastError();  // a CPU-only host has no device: plan->ctas stays 0
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm) {
+    if (variant < -1 || variant >= static_cast<int>(variants().size()))
+        return fail(SAT_ERR_INVALID_VALUE, "unknown variant %d", variant);
+    if (order < 0 || order > 1) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
+    if (ctas_per_sm < 0) return fail(SAT_ERR_INVALID_VALUE, "ctas_per_sm < 0");
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_variant = variant;
+    g_order = order;
+    g_ctas_per_sm = ctas_per_sm;
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_set_max_ctas(int max_ctas) {
+    if (max_ctas < 0) return fail(SAT_ERR_INVALID_VALUE, "max_ctas < 0");
+    std::lock_guard<std::mutex> lk(g_mu);
+    g_max_ctas = max_ctas;
+    return SAT_OK;
+}
+
+SAT_API int sat_num_variants(void) { return static_cast<int>(variants().size()); }
+
+SAT_API sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* tile_cols) {
+    if (variant < 0 || variant >= static_cast<int>(variants().size()))
+        return fail(SAT_ERR_INVALID_VALUE, "unknown variant %d", variant);
+    if (tile_rows) *tile_rows = variants()[variant].TR;
+    if (tile_cols) *tile_cols = variants()[variant].TC;
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out, void* stream) {
+    if (R <= 0 || C <= 0 || R * C > (int64_t(1) << 30) || !out || order < 0 || order > 1)
+        return fail(SAT_ERR_INVALID_VALUE, "bad args");
+    const int64_t n = R * C;
+    int blocks = static_cast<int>((n + 255) / 256);
+    if (blocks > 4096) blocks = 4096;
+    sat::tile_order_kernel<<<blocks, 256, 0, static_cast<cudaStream_t>(stream)>>>(static_cast<int>(R),
+                                                                                  static_cast<int>(C), order, out);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "tile_order_kernel");
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_release_workspaces(void) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    int cur = 0;
+    cudaGetDevice(&cur);
+    for (auto& kv : g_ws) {
+        Workspace* w = kv.second;
+        cudaSetDevice(w->dev);
+        cudaStreamSynchronize(w->stream);
+        if (w->slots) cudaFree(w->slots);
+        if (w->scratch) cudaFree(w->scratch);
+        if (w->ctrl) cudaFree(w->ctrl);
+        delete w;
+    }
+    g_ws.clear();
+    for (auto& kv : g_staging) {
+        cudaSetDevice(kv.first);
+        if (kv.second.buf) cudaFree(kv.second.buf);
+        if (kv.second.h2d) cudaStreamDestroy(kv.second.h2d);
+        if (kv.second.d2h) cudaStreamDestroy(kv.second.d2h);
+    }
+    g_staging.clear();
+    cudaSetDevice(cur);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "release");
+    return SAT_OK;
+}
+
+SAT_API const char* sat_status_string(sat_status_t s) {
+    switch (s) {
+        case SAT_OK: return "SAT_OK";
+        case SAT_ERR_INVALID_VALUE: return "SAT_ERR_INVALID_VALUE";
+        case SAT_ERR_MISALIGNED: return "SAT_ERR_MISALIGNED";
+        case SAT_ERR_UNSUPPORTED: return "SAT_ERR_UNSUPPORTED";
+        case SAT_ERR_OUT_OF_MEMORY: return "SAT_ERR_OUT_OF_MEMORY";
+        case SAT_ERR_CUDA: return "SAT_ERR_CUDA";
+        case SAT_ERR_NCCL: return "SAT_ERR_NCCL";
+    }
+    return "SAT_ERR_UNKNOWN";
+}
+
+SAT_API const char* sat_last_error_detail(void) { return g_detail.c_str(); }
+
+SAT_API int sat_version(void) { return SAT_VERSION; }

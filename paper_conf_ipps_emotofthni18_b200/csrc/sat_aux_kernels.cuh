@@ -1,0 +1,84 @@
+// sat_aux_kernels.cuh -- the multi-GPU strip-carry kernels (not in the paper; BASELINE.json
+// north_star): strip column sums and the carry row of a rank.  Deterministic summation orders.
+#pragma once
+
+#include "sat_device.cuh"
+
+namespace sat {
+
+// Partial column sums: block (x, y) sums rows [y*seg, min((y+1)*seg, rows)) of columns
+// [x*256, x*256+256) into partial[y][col].  One thread per column: every warp reads 128 contiguous
+// bytes per row (coalesced); 8 independent rows in flight per thread.
+template <typename V>
+__global__ void __launch_bounds__(256) colsum_partial_kernel(const V* __restrict__ src, V* __restrict__ partial,
+                                                              int64_t rows, int64_t cols, int64_t pitch,
+                                                              int64_t seg) {
+    const int64_t j = static_cast<int64_t>(blockIdx.x) * 256 + threadIdx.x;
+    if (j >= cols) return;
+    const int64_t r0 = static_cast<int64_t>(blockIdx.y) * seg;
+    int64_t r1 = r0 + seg;
+    if (r1 > rows) r1 = rows;
+    V acc[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) acc[u] = V(0);
+    int64_t i = r0;
+    for (; i + 8 <= r1; i += 8) {
+#pragma unroll
+        for (int u = 0; u < 8; ++u) acc[u] = acc[u] + __ldcs(src + (i + u) * pitch + j);
+    }
+    for (; i < r1; ++i) acc[0] = acc[0] + __ldcs(src + i * pitch + j);
+    V tot = V(0);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) tot = tot + acc[u];
+    partial[static_cast<int64_t>(blockIdx.y) * cols + j] = tot;
+}
+
+// colsum[j] = sum over segments y = 0, 1, ... of partial[y][j] (ascending y).
+template <typename V>
+__global__ void colsum_reduce_kernel(const V* __restrict__ partial, V* __restrict__ colsum, int64_t cols,
+                                     int nseg) {
+    const int64_t j = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+    if (j >= cols) return;
+    V acc = V(0);
+    for (int y = 0; y < nseg; ++y) acc = acc + partial[static_cast<int64_t>(y) * cols + j];
+    colsum[j] = acc;
+}
+
+// Carry row of `rank`: C[j] = sum_{g<rank} gathered[g][j] (ascending g), carry = inclusive
+// row-wise prefix of C.  One CTA of 1024 threads; thread t owns a contiguous chunk.
+template <typename V>
+__global__ void __launch_bounds__(1024) carry_prefix_kernel(const V* __restrict__ gathered, int rank, int64_t cols,
+                                                             V* __restrict__ carry) {
+    __shared__ V warp_tot[32];
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    const int64_t chunk = (cols + 1023) / 1024;
+    const int64_t j0 = t * chunk;
+    int64_t j1 = j0 + chunk;
+    if (j1 > cols) j1 = cols;
+    auto C = [&](int64_t j) {
+        V c = V(0);
+        for (int g = 0; g < rank; ++g) c = c + gathered[static_cast<int64_t>(g) * cols + j];
+        return c;
+    };
+    V mine = V(0);
+    for (int64_t j = j0; j < j1; ++j) mine = mine + C(j);
+    // block exclusive scan of the chunk totals (warp scan, then scan of warp totals)
+    V incl = warp_inclusive_scan(mine, lane);
+    if (lane == 31) warp_tot[warp] = incl;
+    __syncthreads();
+    if (warp == 0) {
+        V x = warp_tot[lane];
+        x = warp_inclusive_scan(x, lane);
+        warp_tot[lane] = x;
+    }
+    __syncthreads();
+    const V up = __shfl_up_sync(kFull, incl, 1);
+    V run = (lane == 0) ? V(0) : up;  // exclusive prefix within the warp
+    if (warp > 0) run = warp_tot[warp - 1] + run;
+    for (int64_t j = j0; j < j1; ++j) {
+        run = run + C(j);
+        carry[j] = run;
+    }
+}
+
+}  // namespace sat

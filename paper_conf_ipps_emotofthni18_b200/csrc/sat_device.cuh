@@ -1,0 +1,150 @@
+// sat_device.cuh -- sm_100a device primitives for libsat: TMA 2-D tile moves with mbarriers,
+// relaxed gpu-scope status words, warp scans.  No SAT-specific logic here (see sat_kernel.cuh).
+#pragma once
+
+#include <cstdint>
+#include <cuda.h>  // CUtensorMap (header only; the driver entry point is resolved at run time)
+#include <cuda_runtime.h>
+
+namespace sat {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// ------------------------------------------------------------------ element arithmetic
+// int32 SAT is computed in uint32 (two's-complement wraparound, R1); fp32 in IEEE fp32.
+__device__ __forceinline__ uint32_t to_bits(uint32_t v) { return v; }
+__device__ __forceinline__ uint32_t to_bits(float v) { return __float_as_uint(v); }
+template <typename V> __device__ __forceinline__ V from_bits(uint32_t b);
+template <> __device__ __forceinline__ uint32_t from_bits<uint32_t>(uint32_t b) { return b; }
+template <> __device__ __forceinline__ float from_bits<float>(uint32_t b) { return __uint_as_float(b); }
+
+// Warp prefix-sum algorithm of P:118-124 (Kogge-Stone, log2(32) = 5 shuffle steps; the "a[i+2^j]"
+// of P:124 is read as a[i-2^j], reading R15).  Inclusive; lane 31 ends with the warp total.
+template <typename V>
+__device__ __forceinline__ V warp_inclusive_scan(V x, int lane) {
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        V y = __shfl_up_sync(kFull, x, d);
+        if (lane >= d) x = x + y;
+    }
+    return x;
+}
+
+template <typename V>
+__device__ __forceinline__ V warp_sum(V x) {
+#pragma unroll
+    for (int d = 16; d >= 1; d >>= 1) x = x + __shfl_xor_sync(kFull, x, d);
+    return x;
+}
+
+// ------------------------------------------------------------------ shared memory / mbarrier
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "SAT_WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra SAT_WAIT_%=;\n}" ::"r"(smem_addr(bar)),
+        "r"(parity)
+        : "memory");
+}
+
+// ------------------------------------------------------------------ TMA (cp.async.bulk.tensor)
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+// 2-D tile global -> shared, completion signalled on `bar` as transaction bytes.  Out-of-bounds
+// box elements are zero-filled (partial edge tiles, R2).
+__device__ __forceinline__ void tma_load_2d(void* smem_dst, const CUtensorMap* map, uint64_t* bar, int x, int y,
+                                            uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1, {%2, %3}], [%4], %5;" ::"r"(smem_addr(smem_dst)),
+        "l"(map), "r"(x), "r"(y), "r"(smem_addr(bar)), "l"(policy)
+        : "memory");
+}
+
+// 2-D tile shared -> global; out-of-bounds box elements are not written (edge tiles, pitch pad).
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* smem_src, int x, int y) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(map), "r"(x),
+                 "r"(y), "r"(smem_addr(smem_src))
+                 : "memory");
+}
+
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// Generic-proxy smem writes -> visible to the async proxy (the TMA store that follows).
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+__device__ __forceinline__ void prefetch_tensormap(const CUtensorMap* map) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
+}
+
+// ------------------------------------------------------------------ gpu-scope status words
+// A status word is 64 bits: high 32 = (epoch << 2) | kind, low 32 = value bits.  One aligned
+// 64-bit access is single-copy atomic, so value and status can never tear; relaxed gpu-scope
+// accesses go to L2 (coherent point for all SMs) and need no fence (R11).
+__device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t a) {
+    asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(a) : "memory");
+}
+__device__ __forceinline__ void st_relaxed2(uint64_t* p, uint64_t a, uint64_t b) {
+    asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
+    uint64_t a;
+    asm volatile("ld.relaxed.gpu.global.b64 %0, [%1];" : "=l"(a) : "l"(p) : "memory");
+    return a;
+}
+__device__ __forceinline__ void ld_relaxed2(const uint64_t* p, uint64_t& a, uint64_t& b) {
+    asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+
+template <int E>
+__device__ __forceinline__ void st_words(uint64_t* p, const uint64_t (&w)[E]) {
+    if constexpr (E == 1) {
+        st_relaxed(p, w[0]);
+    } else {
+#pragma unroll
+        for (int e = 0; e < E; e += 2) st_relaxed2(p + e, w[e], w[e + 1]);
+    }
+}
+
+template <int E>
+__device__ __forceinline__ void ld_words(const uint64_t* p, uint64_t (&w)[E]) {
+    if constexpr (E == 1) {
+        w[0] = ld_relaxed(p);
+    } else {
+#pragma unroll
+        for (int e = 0; e < E; e += 2) ld_relaxed2(p + e, w[e], w[e + 1]);
+    }
+}
+
+}  // namespace sat

@@ -1,0 +1,102 @@
+"""The C-ABI library loads and exports every symbol include/sat.h declares; host-side argument
+handling that needs no GPU.  CPU only: no compute call reaches a kernel here."""
+import ctypes
+import re
+from pathlib import Path
+
+import pytest
+
+ROOT = Path(__file__).resolve().parent.parent
+HEADER = ROOT / "include" / "sat.h"
+
+
+@pytest.fixture(scope="module")
+def sat():
+    import build_native
+
+    build_native.build_libsat()
+    import paper_conf_ipps_emotofthni18_b200 as sat
+
+    return sat
+
+
+def declared_symbols():
+    text = HEADER.read_text()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    return sorted(set(re.findall(r"\b(sat_[a-z0-9_]+)\s*\(", text)))
+
+
+def test_header_declares_the_north_star_entry_points():
+    names = declared_symbols()
+    for must in ("sat_compute_i32", "sat_compute_f32", "sat_compute_sharded"):
+        assert must in names
+
+
+def test_library_exports_every_declared_symbol(sat):
+    lib = ctypes.CDLL(str(ROOT / "paper_conf_ipps_emotofthni18_b200" / "libsat.so"))
+    for name in declared_symbols():
+        assert hasattr(lib, name), f"libsat.so does not export {name}"
+    from paper_conf_ipps_emotofthni18_b200 import _lib
+
+    assert sorted(_lib.EXPORTS) == declared_symbols()
+
+
+def test_version_and_status_strings(sat):
+    from paper_conf_ipps_emotofthni18_b200 import _lib
+
+    assert sat.version() == 100
+    for code, name in _lib.STATUS_NAMES.items():
+        assert _lib.lib().sat_status_string(code).decode() == name
+
+
+def test_variants_and_tuning(sat):
+    n = sat.num_variants()
+    assert n >= 1
+    shapes = [sat.variant_info(v) for v in range(n)]
+    assert all(tc == 128 and tr % 32 == 0 for tr, tc in shapes)
+    with pytest.raises(sat.SatError):
+        sat.variant_info(n)
+    with pytest.raises(sat.SatError):
+        sat.set_tuning(n, 0, 0)
+    with pytest.raises(sat.SatError):
+        sat.set_tuning(-1, 2, 0)
+    sat.set_tuning(-1, 0, 0)
+    sat.set_max_ctas(0)
+
+
+def test_argument_validation_without_gpu(sat):
+    from paper_conf_ipps_emotofthni18_b200 import _lib
+
+    L = _lib.lib()
+    # empty problems are no-ops (no CUDA call needed)
+    assert L.sat_compute(0, None, None, 0, 5, 5, None, None) == 0
+    assert L.sat_compute(1, None, None, 7, 0, 0, None, None) == 0
+    # bad sizes are rejected before any CUDA call
+    assert L.sat_compute(0, 16, 16, 4, 8, 7, None, None) == 1  # pitch < cols
+    assert L.sat_compute(0, 16, 16, -1, 8, 8, None, None) == 1
+    assert L.sat_compute(7, 16, 16, 4, 8, 8, None, None) == 1  # unknown dtype
+    assert L.sat_compute(0, 18, 1 << 20, 4, 8, 8, None, None) == 2  # misaligned
+    assert L.sat_compute(0, 1 << 20, (1 << 20) + 16, 4, 8, 8, None, None) == 1  # partial overlap
+    assert b"overlap" in L.sat_last_error_detail()
+    assert L.sat_compute_host(0, None, None, 3, 4, 2, None) == 1
+
+
+def test_plan_shapes(sat):
+    p = sat.query_plan(sat.SAT_INT32, 1000, 1000, 1024, 1 << 20, 1 << 21)
+    tr, tc = p["tile_rows"], p["tile_cols"]
+    assert p["tiles"] == -(-1000 // tr) * -(-1000 // tc)
+    assert p["tma"] == 1
+    assert p["aux_bytes"] == p["tiles"] * (tr + tc + 1) * 8
+    assert sat.query_plan(sat.SAT_INT32, 1000, 1000, 1001, 1 << 20, 1 << 21)["tma"] == 0  # pitch*4 % 16
+    assert sat.query_plan(sat.SAT_INT32, 10, 10, 12, (1 << 20) + 4, 1 << 21)["tma"] == 0  # pointer % 16
+
+
+def test_strip_bounds_cover_rows_exactly(sat):
+    for rows in [0, 1, 7, 64, 65536, 65537]:
+        for world in [1, 2, 3, 8]:
+            parts = [sat.strip_bounds(rows, world, r) for r in range(world)]
+            assert sum(n for _, n in parts) == rows
+            pos = 0
+            for r0, n in parts:
+                assert n >= 0 and (n == 0 or r0 == pos)
+                pos += n
