@@ -94,6 +94,14 @@ def build_libsat(force: bool = False, extra: list[str] | None = None, out: Path 
     return out
 
 
+def build_stats(force: bool = False) -> Path:
+    """Instrumented libsat (per-CTA phase counters, sat_debug_stats) for tools/stats.py."""
+    out = PKG / "libsat_stats.so"
+    if force or _stale(out, libsat_sources()):
+        build_libsat(extra=["-DSAT_STATS=1"], out=out)
+    return out
+
+
 def build_all(force: bool = False) -> None:
     build_oracle(force)
     build_satgen(force)

@@ -154,6 +154,11 @@ sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* tile_col
  * out: device int32[2*R*C], out[2s] = I, out[2s+1] = J of serial s. */
 sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out, void* stream);
 
+/* Test/tuning hook: per-CTA phase counters (cycles, look-back steps) of the most recent launch.
+ * out: host int64[max_ctas * n_stats].  Only libsat_stats.so (built with -DSAT_STATS=1) records
+ * them; the production library returns SAT_ERR_UNSUPPORTED. */
+sat_status_t sat_debug_stats(int64_t* out, int max_ctas, int* n_ctas, int* n_stats);
+
 /* Free every cached workspace and staging buffer (synchronises the devices that own them). */
 sat_status_t sat_release_workspaces(void);
 

@@ -6,10 +6,12 @@ no fallback: if libsat.so is missing or fails to load, importing the binding rai
 from __future__ import annotations
 
 import ctypes
+import os
 from pathlib import Path
 
 _HERE = Path(__file__).resolve().parent
-LIB_PATH = _HERE / "libsat.so"
+# SAT_LIB may point at an instrumented build (libsat_stats.so, tools/stats.py); never a fallback.
+LIB_PATH = Path(os.environ["SAT_LIB"]) if os.environ.get("SAT_LIB") else _HERE / "libsat.so"
 
 SAT_OK = 0
 SAT_INT32, SAT_FLOAT32 = 0, 1
@@ -22,7 +24,7 @@ STATUS_NAMES = {
 EXPORTS = (
     "sat_compute_i32", "sat_compute_f32", "sat_compute", "sat_compute_host", "sat_strip_colsum",
     "sat_carry_prefix", "sat_comm_get_unique_id", "sat_comm_init", "sat_comm_destroy", "sat_compute_sharded",
-    "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order",
+    "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order", "sat_debug_stats",
     "sat_release_workspaces", "sat_status_string", "sat_last_error_detail", "sat_version",
 )
 
@@ -62,6 +64,7 @@ def _declare(lib):
         "sat_num_variants": [],
         "sat_variant_info": [_int, ctypes.POINTER(_i32), ctypes.POINTER(_i32)],
         "sat_debug_tile_order": [_i64, _i64, _int, _vp, _vp],
+        "sat_debug_stats": [_vp, _int, ctypes.POINTER(_int), ctypes.POINTER(_int)],
         "sat_release_workspaces": [],
         "sat_status_string": [_int],
         "sat_last_error_detail": [],

@@ -17,6 +17,7 @@
 #include "sat.h"
 #include "sat_aux_kernels.cuh"
 #include "sat_kernel.cuh"
+#include "sat_ws_kernel.cuh"
 
 #if defined(SAT_HAVE_NCCL_H)
 #include <nccl.h>
@@ -64,35 +65,54 @@ struct Variant {
     PrepareFn prepare[2];  // [dtype]
 };
 
-template <typename V, typename Cfg, bool TMA, bool CARRY>
-void* kernel_ptr() {
-    return reinterpret_cast<void*>(&sat::sat_tiles_kernel<V, Cfg, TMA, CARRY>);
+// Kernel family traits: the classic kernel (sat_kernel.cuh, TileCfg) and the warp-specialised
+// kernel (sat_ws_kernel.cuh, WsCfg) share one launch interface.
+template <typename Cfg>
+struct Family;
+
+template <int TR, int TC, int NW, int ST>
+struct Family<sat::TileCfg<TR, TC, NW, ST>> {
+    using Cfg = sat::TileCfg<TR, TC, NW, ST>;
+    static constexpr int threads = NW * 32;
+    template <typename V>
+    static constexpr size_t smem() { return sizeof(sat::Smem<V, Cfg>); }
+    template <typename V, bool TMA, bool CARRY>
+    static void* kernel() { return reinterpret_cast<void*>(&sat::sat_tiles_kernel<V, Cfg, TMA, CARRY>); }
+};
+
+template <int TR, int NW, int ST, int NT>
+struct Family<sat::WsCfg<TR, NW, ST, NT>> {
+    using Cfg = sat::WsCfg<TR, NW, ST, NT>;
+    static constexpr int threads = Cfg::THREADS;
+    template <typename V>
+    static constexpr size_t smem() { return sizeof(sat::WsSmem<V, Cfg>); }
+    template <typename V, bool TMA, bool CARRY>
+    static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
+};
+
+template <typename V, typename F>
+void* pick_kernel(bool tma, bool carry) {
+    return tma ? (carry ? F::template kernel<V, true, true>() : F::template kernel<V, true, false>())
+               : (carry ? F::template kernel<V, false, true>() : F::template kernel<V, false, false>());
 }
 
 template <typename V, typename Cfg>
 cudaError_t launch_variant(bool tma, bool carry, dim3 grid, cudaStream_t st, const CUtensorMap& mi,
                            const CUtensorMap& mo, const void* params) {
+    using F = Family<Cfg>;
     const KParams<V>& p = *static_cast<const KParams<V>*>(params);
-    const size_t smem = sizeof(sat::Smem<V, Cfg>);
-    const dim3 block(Cfg::NW * 32);
-    if (tma) {
-        if (carry) sat::sat_tiles_kernel<V, Cfg, true, true><<<grid, block, smem, st>>>(mi, mo, p);
-        else sat::sat_tiles_kernel<V, Cfg, true, false><<<grid, block, smem, st>>>(mi, mo, p);
-    } else {
-        if (carry) sat::sat_tiles_kernel<V, Cfg, false, true><<<grid, block, smem, st>>>(mi, mo, p);
-        else sat::sat_tiles_kernel<V, Cfg, false, false><<<grid, block, smem, st>>>(mi, mo, p);
-    }
-    return cudaGetLastError();
+    void* args[] = {const_cast<CUtensorMap*>(&mi), const_cast<CUtensorMap*>(&mo), const_cast<KParams<V>*>(&p)};
+    return cudaLaunchKernel(pick_kernel<V, F>(tma, carry), grid, dim3(F::threads), args, F::template smem<V>(), st);
 }
 
 template <typename V, typename Cfg>
 cudaError_t prepare_variant(bool tma, bool carry, int* occupancy) {
-    void* k = tma ? (carry ? kernel_ptr<V, Cfg, true, true>() : kernel_ptr<V, Cfg, true, false>())
-                  : (carry ? kernel_ptr<V, Cfg, false, true>() : kernel_ptr<V, Cfg, false, false>());
-    const int smem = static_cast<int>(sizeof(sat::Smem<V, Cfg>));
+    using F = Family<Cfg>;
+    void* k = pick_kernel<V, F>(tma, carry);
+    const int smem = static_cast<int>(F::template smem<V>());
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy, k, Cfg::NW * 32, smem);
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy, k, F::threads, smem);
 }
 
 template <typename Cfg>
@@ -102,7 +122,7 @@ Variant make_variant() {
     v.TC = Cfg::TC;
     v.NW = Cfg::NW;
     v.STAGES = Cfg::STAGES;
-    v.smem = sizeof(sat::Smem<uint32_t, Cfg>);
+    v.smem = Family<Cfg>::template smem<uint32_t>();
     v.launch[SAT_INT32] = &launch_variant<uint32_t, Cfg>;
     v.launch[SAT_FLOAT32] = &launch_variant<float, Cfg>;
     v.prepare[SAT_INT32] = &prepare_variant<uint32_t, Cfg>;
@@ -112,12 +132,12 @@ Variant make_variant() {
 
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
-        make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 0: 32 KiB tiles, 2 stages
-        make_variant<sat::TileCfg<64, 128, 8, 3>>(),   // 1: 32 KiB tiles, 3 stages
-        make_variant<sat::TileCfg<32, 128, 8, 3>>(),   // 2: 16 KiB tiles, 3 stages
-        make_variant<sat::TileCfg<128, 128, 8, 2>>(),  // 3: 64 KiB tiles (the paper's W=128), 2 stages
-        make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 4: 64 KiB tiles, 512 threads
-        make_variant<sat::TileCfg<32, 128, 8, 4>>(),   // 5: 16 KiB tiles, 4 stages
+        make_variant<sat::WsCfg<128, 16, 3, 2>>(),  // 0: warp-specialised, 64 KiB tiles, 3 stages
+        make_variant<sat::WsCfg<128, 16, 3, 1>>(),  // 1: ... one tile in flight per walker
+        make_variant<sat::WsCfg<64, 16, 6, 2>>(),   // 2: warp-specialised, 32 KiB tiles, 6 stages
+        make_variant<sat::WsCfg<64, 8, 6, 2>>(),    // 3: ... 8 compute warps
+        make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 4: classic, 32 KiB tiles, 2 stages
+        make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 5: classic, 64 KiB tiles, 512 threads
     };
     return vs;
 }
@@ -132,7 +152,7 @@ int g_max_ctas = 0;
 int auto_variant(int64_t rows, int64_t cols) {
     (void)cols;
     (void)rows;
-    return 0;
+    return 1;  // best measured at 32K x 32K (tools/sweep_variants.py)
 }
 
 // ------------------------------------------------------------------ device info caches
@@ -178,10 +198,13 @@ struct Workspace {
     uint64_t* slots = nullptr;
     size_t slot_words = 0;
     uint64_t calls = 0;
+    long long* stats = nullptr;  // SAT_STATS builds: [ctas][kNumStats] of the last launch
+    int stats_ctas = 0;
     void* scratch = nullptr;  // colsum partials etc.
     size_t scratch_bytes = 0;
 };
 std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
+Workspace* g_last_stats = nullptr;
 
 sat_status_t reset_ctrl(Workspace* w) {
     Ctrl init{0u, 0u, 1u, 0u};
@@ -385,6 +408,17 @@ sat_status_t compute_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ro
     p.corner_slots = w->slots + static_cast<size_t>(pl.ntiles) * (v.TR + v.TC);
     p.ctrl = w->ctrl;
     p.carry = static_cast<const uint32_t*>(carry);
+    p.stats = nullptr;
+#if SAT_STATS
+    if (w->stats_ctas < grid) {
+        if (w->stats) cudaFree(w->stats);
+        SAT_CUDA(cudaMalloc(&w->stats, static_cast<size_t>(grid) * sat::kNumStats * 8));
+    }
+    w->stats_ctas = static_cast<int>(grid);
+    SAT_CUDA(cudaMemsetAsync(w->stats, 0, static_cast<size_t>(grid) * sat::kNumStats * 8, st));
+    p.stats = w->stats;
+    g_last_stats = w;
+#endif
     cudaError_t e = v.launch[dt](pl.tma, carry != nullptr, dim3(static_cast<unsigned>(grid)), st, mi, mo, &p);
     if (e != cudaSuccess) return cuda_fail(e, "sat_tiles_kernel launch");
     w->calls++;
@@ -772,6 +806,23 @@ SAT_API sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32
     return SAT_OK;
 }
 
+SAT_API sat_status_t sat_debug_stats(int64_t* out, int max_ctas, int* n_ctas, int* n_stats) {
+#if SAT_STATS
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (!g_last_stats || !out || !n_ctas || !n_stats) return fail(SAT_ERR_INVALID_VALUE, "no stats");
+    Workspace* w = g_last_stats;
+    const int n = w->stats_ctas < max_ctas ? w->stats_ctas : max_ctas;
+    SAT_CUDA(cudaStreamSynchronize(w->stream));
+    SAT_CUDA(cudaMemcpy(out, w->stats, static_cast<size_t>(n) * sat::kNumStats * 8, cudaMemcpyDeviceToHost));
+    *n_ctas = n;
+    *n_stats = sat::kNumStats;
+    return SAT_OK;
+#else
+    (void)out; (void)max_ctas; (void)n_ctas; (void)n_stats;
+    return fail(SAT_ERR_UNSUPPORTED, "libsat built without SAT_STATS");
+#endif
+}
+
 SAT_API sat_status_t sat_release_workspaces(void) {
     std::lock_guard<std::mutex> lk(g_mu);
     int cur = 0;
@@ -783,9 +834,11 @@ SAT_API sat_status_t sat_release_workspaces(void) {
         if (w->slots) cudaFree(w->slots);
         if (w->scratch) cudaFree(w->scratch);
         if (w->ctrl) cudaFree(w->ctrl);
+        if (w->stats) cudaFree(w->stats);
         delete w;
     }
     g_ws.clear();
+    g_last_stats = nullptr;
     for (auto& kv : g_staging) {
         cudaSetDevice(kv.first);
         if (kv.second.buf) cudaFree(kv.second.buf);

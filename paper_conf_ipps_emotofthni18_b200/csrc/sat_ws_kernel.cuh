@@ -1,0 +1,629 @@
+// sat_ws_kernel.cuh -- warp-specialised single-pass SAT kernel for sm_100a (the production kernel).
+//
+// Same method and same published aggregates as sat_tiles_kernel (sat_kernel.cuh: 1R1W-SKSS-LB of
+// PAPER.md Sec. IV, prefix-form slots, epoch-tagged status words), but the steps of a tile
+// run on dedicated warps so that their latencies overlap.  Measured on B200: with HBM saturated an
+// L2 round trip (a look-back poll) costs ~1-2 us, the same order as one tile's whole compute, so the
+// look-backs must run ahead of the tile they serve.  Roles of a persistent CTA:
+//
+//   loader (1 lane)    SKSS ticket c <- atomicAdd(&c,1) (drawn one tile ahead),
+//                      Fig. 9 serial -> (I,J), TMA 2-D load of T(I,J) into a ring of STAGES
+//                      shared-memory stages (Step 1).
+//   row walker warp    row look-back (Step 2.A.2) and diagonal look-back (Step 3.2,
+//                      P:241) of the CTA's tiles, started as soon as a tile is acquired, several
+//                      tiles per polling round; results -> the tile's stage slots (rp, corner).
+//   column walker warp column look-back (Step 2.B.2); result -> cp.
+//   NW compute warps   local SAT of the tile in registers; local aggregates published
+//                      from the owning lanes (Steps 2.A.1, 2.B.1); once the walks are in, the
+//                      inclusive aggregates GRS/GCS/GS from the same lanes (Steps 2.A.3, 2.B.3, 3.1,
+//                      3.3) and the Step 4 correction (rule P:150) written to the stage.
+//   storer (1 lane)    TMA 2-D store of GSAT(I,J) (Step 4), two in flight; frees stages.
+//
+// Hand-offs are mbarriers per stage: acq (tile id written), full (TMA bytes landed, or "no more
+// tiles"), rowwalk / colwalk (carries in smem), result (GSAT in smem, NW arrivals), empty (stage read
+// by its TMA store).  Each completes once per use of its stage (tile k: stage k % STAGES, parity
+// (k / STAGES) & 1, tracked incrementally by Slot).  Forward progress: tiles are acquired in serial
+// order; every role handles its CTA's tiles in that order; a walk only waits on tiles with smaller
+// serial numbers, whose local aggregates depend on nothing but their own data.
+#pragma once
+
+#include "sat_kernel.cuh"
+
+namespace sat {
+
+// Stats builds (-DSAT_STATS=1): per-CTA counters in shared memory, role-tagged slots.
+enum WsStat {
+    kWsTiles = 0, kWsFullWait, kWsLocal, kWsWalkWait, kWsFinish, kWsRowRounds, kWsColRounds,
+    kWsStResultWait, kWsStStore, kWsLdIssue, kWsLdEmptyWait, kWsBandBar, kWsRowTiles, kWsColTiles
+};
+#if SAT_STATS
+__shared__ unsigned long long ws_stats[kNumStats];
+#define WS_ST(k, v) atomicAdd(&ws_stats[k], static_cast<unsigned long long>(v))
+#else
+#define WS_ST(k, v) (void)0
+#endif
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
+}
+
+// One bounded try_wait (the hardware may suspend the thread a while before reporting "not yet").
+__device__ __forceinline__ bool mbar_try(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(ok)
+        : "r"(smem_addr(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+
+// Non-blocking probe of an mbarrier phase.
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(ok)
+        : "r"(smem_addr(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+template <int TR_, int NW_, int STAGES_, int NT_>
+struct WsCfg {
+    static constexpr int TR = TR_, TC = 128, NW = NW_, STAGES = STAGES_;
+    static constexpr int NT = NT_;        // tiles in flight per walker
+    static constexpr int RPW = TR / NW;   // rows per compute-warp band
+    static constexpr int ER = TR / 32;    // row-vector elements per walker lane
+    static constexpr int EC = TC / 32;    // column-vector elements per walker lane
+    static constexpr int ROW_WARP = NW, COL_WARP = NW + 1, STORE_WARP = NW + 2, LOAD_WARP = NW + 3;
+    static constexpr int THREADS = (NW + 4) * 32;
+    static constexpr int MINB = 1;
+    static_assert(TR % NW == 0 && TR % 32 == 0, "tile shape");
+    static_assert(RPW % 2 == 0, "row slots are published in pairs");
+    static_assert(ER == 1 || ER % 2 == 0, "row vector split");
+    static_assert(STAGES >= 2 && STAGES <= 8 && NT >= 1, "ring");
+};
+
+template <typename V, typename Cfg>
+struct WsSmem {
+    alignas(1024) V stage[Cfg::STAGES][Cfg::TR * Cfg::TC];
+    alignas(16) V band[2][Cfg::NW][Cfg::TC];
+    alignas(16) V rp[Cfg::STAGES][Cfg::TR];  // row carry    prefix_i GRS(I,J-1)
+    alignas(16) V cp[Cfg::STAGES][Cfg::TC];  // column carry prefix_j GCS(I-1,J)
+    V corner[Cfg::STAGES];                   // GS(I-1,J-1)
+    alignas(8) uint64_t acq[Cfg::STAGES];
+    uint64_t full[Cfg::STAGES];
+    uint64_t rowwalk[Cfg::STAGES];
+    uint64_t colwalk[Cfg::STAGES];
+    uint64_t result[Cfg::STAGES];
+    uint64_t empty[Cfg::STAGES];
+    alignas(16) TileInfo info[Cfg::STAGES];
+    uint32_t epoch;
+    int end_n;  // index of the end marker once the loader has drawn an invalid ticket, else INT_MAX
+};
+
+// Position of tile k in the stage ring: stage s = k % STAGES, barrier phase parity (k / STAGES) & 1,
+// advanced incrementally (no division in the loops).
+template <int STAGES>
+struct Slot {
+    int k = 0, s = 0;
+    uint32_t ph = 0;
+    __device__ __forceinline__ void next() {
+        ++k;
+        if (++s == STAGES) { s = 0; ph ^= 1u; }
+    }
+};
+
+// Walkers only wait for their next tile's acquisition; once the loader has drawn the end marker they
+// stop.  Returns false when tile k will never exist.
+template <typename V, typename Cfg>
+__device__ __forceinline__ bool wait_acquired(WsSmem<V, Cfg>& sm, int s, uint32_t parity, int k) {
+    while (!mbar_try(&sm.acq[s], parity))
+        if (k >= *reinterpret_cast<volatile int*>(&sm.end_n)) return false;
+    return true;
+}
+
+// One round of a 2-deep windowed vector look-back (Steps 2.A.2 / 2.B.2): the lane's E elements,
+// predecessor position `pos` (and pos-1) along the walk, words already loaded.  Consumes ready
+// predecessors in order, stops at the first not-ready one.  Returns true if it made progress.
+template <typename V, int E>
+__device__ __forceinline__ bool lb_consume(uint32_t& pending, int& pos, V (&acc)[E], const uint64_t (&w0)[E],
+                                           const uint64_t (&w1)[E], bool have1, uint32_t epoch) {
+    bool progress = false;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+        if (!pending || (h == 1 && !have1)) break;
+        const uint64_t(&w)[E] = h == 0 ? w0 : w1;
+        bool ok = true;
+#pragma unroll
+        for (int e = 0; e < E; ++e)
+            if (((pending >> e) & 1u) && !word_ready(w[e], epoch)) ok = false;
+        if (!ok) break;
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+            if ((pending >> e) & 1u) {
+                acc[e] = acc[e] + from_bits<V>(static_cast<uint32_t>(w[e]));
+                if (word_kind(w[e]) == kIncl) pending &= ~(1u << e);
+            }
+        }
+        pos -= 1;
+        progress = true;
+    }
+    return progress;
+}
+
+template <typename V, typename Cfg, bool ROW>
+__device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, STAGES = Cfg::STAGES;
+    constexpr int E = ROW ? Cfg::ER : Cfg::EC;
+    constexpr int NT = Cfg::NT;
+    struct Walk {
+        int active, s, I, J, pos;
+        uint32_t pend;
+        V acc[E];
+        V dacc;
+        int dbase, ddone;
+    };
+    Walk wk[NT];
+#pragma unroll
+    for (int w = 0; w < NT; ++w) wk[w].active = 0;
+    Slot<STAGES> next;
+    bool ended = false;
+    int steps = 0;
+    while (true) {
+        // ---- take newly acquired tiles into free walk slots (block only when nothing is in flight)
+#pragma unroll
+        for (int w = 0; w < NT; ++w) {
+            if (wk[w].active || ended) continue;
+            bool busy = false;
+#pragma unroll
+            for (int v2 = 0; v2 < NT; ++v2) busy = busy || wk[v2].active;
+            bool got;
+            if (busy) {
+                got = mbar_test(&sm.acq[next.s], next.ph);
+                if (!got && next.k >= *reinterpret_cast<volatile int*>(&sm.end_n)) ended = true;
+            } else {
+                got = wait_acquired(sm, next.s, next.ph, next.k);
+                if (!got) ended = true;
+            }
+            if (!got) continue;
+            const TileInfo ti = sm.info[next.s];
+            if (ti.t >= p.ntiles) {
+                ended = true;
+                continue;
+            }
+            Walk& x = wk[w];
+            x.active = 1;
+            x.s = next.s;
+            x.I = ti.I;
+            x.J = ti.J;
+            x.pos = ROW ? ti.J - 1 : ti.I - 1;
+            x.pend = (x.pos >= 0) ? ((1u << E) - 1u) : 0u;
+#pragma unroll
+            for (int e = 0; e < E; ++e) x.acc[e] = V(0);
+            x.dacc = V(0);
+            x.dbase = 1;
+            x.ddone = ROW ? (ti.I == 0 || ti.J == 0) : 1;
+            next.next();
+        }
+        bool any = false;
+#pragma unroll
+        for (int w = 0; w < NT; ++w) any = any || wk[w].active;
+        if (!any) {
+            if (ended) break;
+            continue;
+        }
+        // ---- one polling round: issue every load first ...
+        uint64_t w0[NT][E], w1[NT][E], wd[NT];
+#pragma unroll
+        for (int w = 0; w < NT; ++w) {
+            const Walk& x = wk[w];
+            wd[w] = 0;
+            if (!x.active) continue;
+            if (x.pend) {
+                if (ROW) {
+                    const long long base = static_cast<long long>(x.I) * p.C;
+                    ld_words<E>(p.row_slots + (base + x.pos) * TR + lane * E, w0[w]);
+                    if (x.pos >= 1) ld_words<E>(p.row_slots + (base + x.pos - 1) * TR + lane * E, w1[w]);
+                } else {
+                    ld_words<E>(p.col_slots + (static_cast<long long>(x.pos) * p.C + x.J) * TC + lane * E, w0[w]);
+                    if (x.pos >= 1)
+                        ld_words<E>(p.col_slots + (static_cast<long long>(x.pos - 1) * p.C + x.J) * TC + lane * E,
+                                    w1[w]);
+                }
+            }
+            if (ROW && !x.ddone) wd[w] = diag_word(p.corner_slots, x.I, x.J, p.C, x.dbase + lane);
+        }
+        ++steps;
+        // ---- ... then consume them
+        bool progress = false;
+#pragma unroll
+        for (int w = 0; w < NT; ++w) {
+            Walk& x = wk[w];
+            if (!x.active) continue;
+            if (x.pend) progress |= lb_consume<V, E>(x.pend, x.pos, x.acc, w0[w], w1[w], x.pos >= 1, epoch);
+            if (ROW && !x.ddone) {
+                // Step 3.2: GS(I-1,J-1) = GS(I-k,J-k) + sum of GLS of the tiles between
+                const int kk = x.dbase + lane;
+                const bool inrange = (x.I - kk >= 0) && (x.J - kk >= 0);
+                const bool ready = !inrange || word_ready(wd[w], epoch);
+                const unsigned incl = __ballot_sync(kFull, inrange && ready && word_kind(wd[w]) == kIncl);
+                const unsigned notready = __ballot_sync(kFull, !ready);
+                const int f = incl ? (__ffs(incl) - 1) : 32;
+                const unsigned need = (f >= 31) ? kFull : ((2u << f) - 1u);
+                if (!(notready & need)) {
+                    const V val = (inrange && lane <= f) ? from_bits<V>(static_cast<uint32_t>(wd[w])) : V(0);
+                    x.dacc = x.dacc + warp_sum(val);
+                    if (f < 32) x.ddone = 1; else x.dbase += 32;
+                    progress = true;
+                }
+            }
+            if (x.ddone && __all_sync(kFull, x.pend == 0u)) {
+                if (ROW) {
+#pragma unroll
+                    for (int e = 0; e < E; ++e) sm.rp[x.s][lane * E + e] = x.acc[e];
+                    if (lane == 0) sm.corner[x.s] = x.dacc;
+                } else {
+#pragma unroll
+                    for (int e = 0; e < E; ++e) sm.cp[x.s][lane * E + e] = x.acc[e];
+                }
+                __syncwarp();
+                if (lane == 0) {
+                    mbar_arrive(ROW ? &sm.rowwalk[x.s] : &sm.colwalk[x.s]);
+                    WS_ST(ROW ? kWsRowTiles : kWsColTiles, 1);
+                }
+                x.active = 0;
+                progress = true;
+            }
+        }
+        if (!__any_sync(kFull, progress)) __nanosleep(64);
+    }
+    if (lane == 0) WS_ST(ROW ? kWsRowRounds : kWsColRounds, steps);
+}
+
+// Step 1, local SAT, Steps 2.A.1 / 2.B.1 of the tile in stage sl.s into registers `v`.  Returns false
+// at the end marker.
+template <typename V, typename Cfg, bool TMA>
+__device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p, V (&v)[Cfg::RPW][4],
+                                         const Slot<Cfg::STAGES>& sl, int& I, int& J, uint32_t epoch, int warp,
+                                         int lane) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
+    const int s = sl.s;
+    const int row0 = warp * RPW, col0 = lane * 4;
+    SAT_CLK(c0);
+    mbar_wait(&sm.full[s], sl.ph);
+    SAT_CLK(c1);
+    if (warp == 0 && lane == 0) { WS_ST(kWsFullWait, c1 - c0); WS_ST(kWsTiles, 1); }
+    const TileInfo ti = sm.info[s];
+    if (ti.t >= p.ntiles) return false;
+    I = ti.I;
+    J = ti.J;
+    const long long tidx = static_cast<long long>(I) * p.C + J;
+    const int par = sl.k & 1;
+
+    // ---- Step 1 (data in smem, or read from global on the generic path): tile -> registers
+    if constexpr (TMA) {
+        const V* tile = sm.stage[s];
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const uint4 q = *reinterpret_cast<const uint4*>(&tile[(row0 + r) * TC + col0]);
+            v[r][0] = from_bits<V>(q.x); v[r][1] = from_bits<V>(q.y);
+            v[r][2] = from_bits<V>(q.z); v[r][3] = from_bits<V>(q.w);
+        }
+        if (J == p.C - 1) {  // right edge: zero columns >= cols (16-byte TMA granules, reading R2)
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                if (static_cast<long long>(J) * TC + col0 + c >= p.cols) {
+#pragma unroll
+                    for (int r = 0; r < RPW; ++r) v[r][c] = V(0);
+                }
+        }
+    } else {
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const long long gi = static_cast<long long>(I) * TR + row0 + r;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const long long gj = static_cast<long long>(J) * TC + col0 + c;
+                v[r][c] = (gi < p.rows && gj < p.cols) ? p.src[gi * p.pitch + gj] : V(0);
+            }
+        }
+    }
+
+    // ---- local SAT: column prefix inside the warp's band, row scans with the warp prefix-sum
+    //      algorithm, then the SAT rows of the bands above
+#pragma unroll
+    for (int r = 1; r < RPW; ++r)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + v[r - 1][c];
+#pragma unroll
+    for (int r = 0; r < RPW; ++r) {
+        v[r][1] = v[r][1] + v[r][0];
+        v[r][2] = v[r][2] + v[r][1];
+        v[r][3] = v[r][3] + v[r][2];
+        const V incl = warp_inclusive_scan(v[r][3], lane);
+        V excl = __shfl_up_sync(kFull, incl, 1);
+        if (lane == 0) excl = V(0);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + excl;
+    }
+    *reinterpret_cast<uint4*>(&sm.band[par][warp][col0]) =
+        make_uint4(to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
+    SAT_CLK(cb0);
+    named_bar_sync(1, NW * 32);
+    SAT_CLK(cb1);
+    if (warp == 0 && lane == 0) WS_ST(kWsBandBar, cb1 - cb0);
+    {
+        // column-wise exclusive scan of the NW band bottoms, in place, by the first TC compute
+        // threads (one column each); then every warp reads its band's offset in one 16-byte load
+        const int tid = warp * 32 + lane;
+        if (tid < TC) {
+            V b[NW];
+#pragma unroll
+            for (int u = 0; u < NW; ++u) b[u] = sm.band[par][u][tid];
+            V run = V(0);
+#pragma unroll
+            for (int u = 0; u < NW; ++u) {
+                sm.band[par][u][tid] = run;
+                run = run + b[u];
+            }
+        }
+        named_bar_sync(1, NW * 32);
+        const uint4 q = *reinterpret_cast<const uint4*>(&sm.band[par][warp][col0]);
+        const V off[4] = {from_bits<V>(q.x), from_bits<V>(q.y), from_bits<V>(q.z), from_bits<V>(q.w)};
+#pragma unroll
+        for (int r = 0; r < RPW; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + off[c];
+    }
+
+    // ---- Steps 2.A.1 / 2.B.1: local aggregates (prefix form) from the owning lanes: the last column
+    //      (lane 31 of every warp) and the bottom row (last warp).  Edge tiles publish inclusive at
+    //      once: their carry is zero.
+    if (lane == 31) {
+        uint64_t* rs = p.row_slots + tidx * TR + row0;
+        const uint32_t kind = (J == 0) ? kIncl : kLocal;
+#pragma unroll
+        for (int r = 0; r < RPW; r += 2)
+            st_relaxed2(rs + r, pack(epoch, kind, to_bits(v[r][3])), pack(epoch, kind, to_bits(v[r + 1][3])));
+    }
+    if (warp == NW - 1) {
+        uint64_t* cs = p.col_slots + tidx * TC + col0;
+        const uint32_t kind = (I == 0) ? kIncl : kLocal;
+        st_relaxed2(cs, pack(epoch, kind, to_bits(v[RPW - 1][0])), pack(epoch, kind, to_bits(v[RPW - 1][1])));
+        st_relaxed2(cs + 2, pack(epoch, kind, to_bits(v[RPW - 1][2])), pack(epoch, kind, to_bits(v[RPW - 1][3])));
+    }
+    SAT_CLK(c2);
+    if (warp == 0 && lane == 0) WS_ST(kWsLocal, c2 - c1);
+    return true;
+}
+
+// Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 and Step 4 for the tile in stage sl.s whose local SAT is in `v`.
+template <typename V, typename Cfg, bool TMA, bool CARRY>
+__device__ __forceinline__ void ws_finish(WsSmem<V, Cfg>& sm, const KParams<V>& p, V (&v)[Cfg::RPW][4],
+                                          const Slot<Cfg::STAGES>& sl, int I, int J, uint32_t epoch, int warp,
+                                          int lane) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
+    const int s = sl.s;
+    const int row0 = warp * RPW, col0 = lane * 4;
+    const long long tidx = static_cast<long long>(I) * p.C + J;
+    SAT_CLK(c0);
+    mbar_wait(&sm.rowwalk[s], sl.ph);
+    mbar_wait(&sm.colwalk[s], sl.ph);
+    SAT_CLK(c1);
+    if (warp == 0 && lane == 0) WS_ST(kWsWalkWait, c1 - c0);
+    V rt[RPW];
+#pragma unroll
+    for (int r = 0; r < RPW; ++r) rt[r] = sm.rp[s][row0 + r];
+    V cpv[4];
+    {
+        const uint4 q = *reinterpret_cast<const uint4*>(&sm.cp[s][col0]);
+        cpv[0] = from_bits<V>(q.x); cpv[1] = from_bits<V>(q.y); cpv[2] = from_bits<V>(q.z); cpv[3] = from_bits<V>(q.w);
+    }
+    const V corner = sm.corner[s];
+    // inclusive aggregates, from the lanes that hold the local ones
+    if (lane == 31 && J > 0) {
+        uint64_t* rs = p.row_slots + tidx * TR + row0;
+#pragma unroll
+        for (int r = 0; r < RPW; r += 2)
+            st_relaxed2(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + rt[r])),
+                        pack(epoch, kIncl, to_bits(v[r + 1][3] + rt[r + 1])));
+    }
+    if (warp == NW - 1) {
+        if (I > 0) {
+            uint64_t* cs = p.col_slots + tidx * TC + col0;
+            st_relaxed2(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + cpv[0])),
+                        pack(epoch, kIncl, to_bits(v[RPW - 1][1] + cpv[1])));
+            st_relaxed2(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + cpv[2])),
+                        pack(epoch, kIncl, to_bits(v[RPW - 1][3] + cpv[3])));
+        }
+        if (lane == 31) {  // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
+            const V gls = v[RPW - 1][3] + rt[RPW - 1] + cpv[3];
+            st_relaxed(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(corner + gls)));
+        }
+    }
+    // GSAT(I,J) = localSAT + rp[i] + cp[j] + corner (+ carry[j])
+    V colterm[4];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) colterm[c] = cpv[c] + corner;
+    if constexpr (CARRY) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const long long gj = static_cast<long long>(J) * TC + col0 + c;
+            colterm[c] = colterm[c] + (gj < p.cols ? p.carry[gj] : V(0));
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < RPW; ++r)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + (rt[r] + colterm[c]);
+    const bool ragged = !TMA || ((J == p.C - 1) && (p.cols & 3) != 0);
+    if (!ragged) {
+        V* tile = sm.stage[s];
+#pragma unroll
+        for (int r = 0; r < RPW; ++r)
+            *reinterpret_cast<uint4*>(&tile[(row0 + r) * TC + col0]) =
+                make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3]));
+        fence_proxy_async_smem();
+    } else {
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const long long gi = static_cast<long long>(I) * TR + row0 + r;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const long long gj = static_cast<long long>(J) * TC + col0 + c;
+                if (gi < p.rows && gj < p.cols) p.dst[gi * p.pitch + gj] = v[r][c];
+            }
+        }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sm.result[s]);
+    SAT_CLK(c2);
+    if (warp == 0 && lane == 0) WS_ST(kWsFinish, c2 - c1);
+}
+
+template <typename V, typename Cfg, bool TMA, bool CARRY>
+__global__ void __launch_bounds__(Cfg::THREADS, Cfg::MINB)
+sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant__ CUtensorMap map_out,
+              const KParams<V> p) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, STAGES = Cfg::STAGES, RPW = Cfg::RPW;
+    constexpr uint32_t kTileBytes = TR * TC * sizeof(V);
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    WsSmem<V, Cfg>& sm = *reinterpret_cast<WsSmem<V, Cfg>*>(smem_raw);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+#if SAT_STATS
+    if (threadIdx.x < kNumStats) ws_stats[threadIdx.x] = 0ull;
+#endif
+    if (threadIdx.x == 0) {
+        sm.epoch = *reinterpret_cast<volatile unsigned int*>(&p.ctrl->epoch);
+        sm.end_n = 0x7fffffff;
+#pragma unroll
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(&sm.acq[s], 1);
+            mbar_init(&sm.full[s], 1);
+            mbar_init(&sm.rowwalk[s], 1);
+            mbar_init(&sm.colwalk[s], 1);
+            mbar_init(&sm.result[s], NW);
+            mbar_init(&sm.empty[s], 1);
+        }
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const uint32_t epoch = sm.epoch;
+
+    if (warp < NW) {
+        // ================================================================ compute warps
+        V v[RPW][4];
+        for (Slot<STAGES> sl;; sl.next()) {
+            int I, J;
+            if (!ws_local<V, Cfg, TMA>(sm, p, v, sl, I, J, epoch, warp, lane)) break;
+            ws_finish<V, Cfg, TMA, CARRY>(sm, p, v, sl, I, J, epoch, warp, lane);
+        }
+    } else if (warp == Cfg::ROW_WARP) {
+        ws_walker<V, Cfg, true>(sm, p, epoch, lane);
+    } else if (warp == Cfg::COL_WARP) {
+        ws_walker<V, Cfg, false>(sm, p, epoch, lane);
+    } else if (warp == Cfg::STORE_WARP) {
+        // ================================================================ storer (one lane)
+        if (lane == 0) {
+            if constexpr (TMA) prefetch_tensormap(&map_out);
+            int pending = -1;  // stage whose store was issued last and is not yet released
+            for (Slot<STAGES> sl;; sl.next()) {
+                const int s = sl.s;
+                mbar_wait(&sm.acq[s], sl.ph);
+                const TileInfo ti = sm.info[s];  // stays valid until this lane releases the stage
+                if (ti.t >= p.ntiles) break;
+                SAT_CLK(u0);
+                mbar_wait(&sm.result[s], sl.ph);
+                SAT_CLK(u1);
+                WS_ST(kWsStResultWait, u1 - u0);
+                bool stored = false;
+                if constexpr (TMA) {
+                    const bool ragged = (ti.J == p.C - 1) && (p.cols & 3) != 0;
+                    if (!ragged) {
+                        tma_store_2d(&map_out, sm.stage[s], ti.J * TC, ti.I * TR);
+                        bulk_commit();
+                        stored = true;
+                    }
+                }
+                // two stores in flight: release the previous stage once its store has read smem
+                if (pending >= 0) {
+                    if (stored) bulk_wait_read<1>(); else bulk_wait_read<0>();
+                    mbar_arrive(&sm.empty[pending]);
+                }
+                if (stored) {
+                    pending = s;
+                } else {
+                    mbar_arrive(&sm.empty[s]);
+                    pending = -1;
+                }
+                SAT_CLK(u2);
+                WS_ST(kWsStStore, u2 - u1);
+            }
+            if (pending >= 0) {
+                bulk_wait_read<0>();
+                mbar_arrive(&sm.empty[pending]);
+            }
+            if constexpr (TMA) bulk_wait_all();
+            __threadfence();
+            const unsigned int done = atomicAdd(&p.ctrl->exit_count, 1u);
+#if SAT_STATS
+            if (p.stats)
+                for (int k = 0; k < kNumStats; ++k)
+                    p.stats[static_cast<long long>(blockIdx.x) * kNumStats + k] = static_cast<long long>(ws_stats[k]);
+#endif
+            if (done == gridDim.x - 1) {
+                p.ctrl->counter = 0u;
+                p.ctrl->exit_count = 0u;
+                p.ctrl->epoch = (epoch >= kEpochMax) ? 1u : epoch + 1u;
+                __threadfence();
+            }
+        }
+    } else if (lane == 0) {
+        // ================================================================ loader (one lane)
+        const uint64_t policy = TMA ? policy_evict_first() : 0ull;
+        if constexpr (TMA) prefetch_tensormap(&map_in);
+        // the next ticket is drawn right after a load is issued, so its L2 round trip overlaps the
+        // wait for a free stage (a CTA holds at most STAGES+1 tiles)
+        unsigned int ticket = atomicAdd(&p.ctrl->counter, 1u);
+        for (Slot<STAGES> sl;; sl.next()) {
+            const int s = sl.s;
+            if (sl.k >= STAGES) {  // wait until the store of the stage's previous tile has read it
+                SAT_CLK(e0);
+                mbar_wait(&sm.empty[s], sl.ph ^ 1u);
+                SAT_CLK(e1);
+                WS_ST(kWsLdEmptyWait, e1 - e0);
+            }
+            SAT_CLK(t0);
+            const int t = static_cast<int>(ticket);
+            const bool valid = t < p.ntiles;
+            TileInfo ti{t, 0, 0, 0};
+            if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
+            sm.info[s] = ti;
+            if (!valid) *reinterpret_cast<volatile int*>(&sm.end_n) = sl.k;
+            mbar_arrive(&sm.acq[s]);
+            if (TMA && valid) {
+                mbar_arrive_expect_tx(&sm.full[s], kTileBytes);
+                tma_load_2d(sm.stage[s], &map_in, &sm.full[s], ti.J * TC, ti.I * TR, policy);
+            } else {
+                mbar_arrive(&sm.full[s]);  // generic path (data read from global) or end marker
+            }
+            if (valid) ticket = atomicAdd(&p.ctrl->counter, 1u);
+            SAT_CLK(t1);
+            WS_ST(kWsLdIssue, t1 - t0);
+            if (!valid) break;
+        }
+    }
+}
+
+}  // namespace sat

@@ -130,6 +130,15 @@ def test_int32_misaligned_base_uses_generic_path(sat):
     assert_i32_exact(run_sat(sat, a, offset_words=1), a)
 
 
+@pytest.mark.parametrize("cols", [997, 998, 999, 1000, 1001])
+@pytest.mark.parametrize("inplace", [False, True])
+def test_ragged_width_with_pad(sat, cols, inplace):
+    """Row widths that are not a multiple of 4 elements: pad words of a 16-byte-aligned pitch must stay
+    untouched by the TMA path."""
+    a = satgen.gen_host(333, cols, seed=cols, dist="u32")
+    assert_i32_exact(run_sat(sat, a, pitch=1008, inplace=inplace), a)
+
+
 def test_int32_in_place(sat):
     a = satgen.gen_host(1111, 999, seed=8, dist="u32")
     assert_i32_exact(run_sat(sat, a, inplace=True), a)
@@ -212,7 +221,7 @@ def test_error_codes_on_gpu(sat):
     base = t.data_ptr()
     assert L.sat_compute(0, base + 2, base + 8192, 4, 8, 8, None, None) == 2  # MISALIGNED
     assert L.sat_compute(0, base, base + 16, 4, 8, 8, None, None) == 1       # partial overlap
-    with pytest.raises(sat.SatError):
+    with pytest.raises(TypeError):
         sat.sat(torch.zeros((4, 4), dtype=torch.int64, device="cuda"))
 
 
