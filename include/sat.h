@@ -133,6 +133,8 @@ typedef struct {
     int64_t aux_bytes;     /* bytes of per-tile aggregate slots for this shape */
     int32_t variant;       /* kernel variant index */
     int32_t order;         /* 0 = diagonal-major (Fig. 9), 1 = row-major */
+    int32_t family;        /* 1 = warp-specialised kernel (sat_ws_kernel), 0 = classic (sat_tiles_kernel) */
+    int32_t reserved;
 } sat_plan_t;
 
 /* Fill `plan` with what sat_compute would launch for this problem (no launch, no allocation). */

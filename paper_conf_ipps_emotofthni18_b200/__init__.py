@@ -22,6 +22,7 @@ _lib.lib()  # load now: fail loudly at import if the native library is missing
 
 __all__ = [
     "sat", "sat_host", "compute", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "strip_layout", "broadcast_unique_id",
     "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "release_workspaces",
     "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
 ]
@@ -140,6 +141,42 @@ def strip_bounds(rows: int, world: int, rank: int) -> tuple[int, int]:
     return row0, min(h, rows - row0)
 
 
+def broadcast_unique_id(group=None) -> bytes:
+    """Rank 0 of ``group`` draws a 128-byte NCCL unique id (sat_comm_get_unique_id) and the group
+    broadcasts it (over the group's own backend: NCCL needs a CUDA tensor, gloo a CPU one)."""
+    import torch.distributed as dist
+
+    torch = _torch()
+    buf = ctypes.create_string_buffer(128)
+    if dist.get_rank(group) == 0:
+        check(_lib.lib().sat_comm_get_unique_id(buf), "sat_comm_get_unique_id")
+    dev = torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl" else torch.device("cpu")
+    t = torch.tensor(list(buf.raw), dtype=torch.uint8, device=dev)
+    dist.broadcast(t, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+    return bytes(t.cpu().tolist())
+
+
+def strip_layout(rows: int, cols: int, dtype_code: int, group=None) -> tuple[int, int]:
+    """Collective host-side check of a strip partition: every rank passes its own strip height and the
+    common column count / dtype.  Returns (row0 of this rank, total rows).  Raises ValueError on every
+    rank if the ranks disagree on cols or dtype (sat_compute_sharded requires equal cols)."""
+    import torch.distributed as dist
+
+    torch = _torch()
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl" else torch.device("cpu")
+    mine = torch.tensor([rows, cols, dtype_code], dtype=torch.int64, device=dev)
+    allv = [torch.empty_like(mine) for _ in range(world)]
+    dist.all_gather(allv, mine, group=group)
+    table = [tuple(int(x) for x in v.cpu().tolist()) for v in allv]
+    if any(c != table[0][1] or d != table[0][2] for _, c, d in table):
+        raise ValueError(f"strip partition mismatch across ranks: (rows, cols, dtype) = {table}")
+    if any(r < 0 for r, _, _ in table):
+        raise ValueError("negative strip height")
+    row0 = sum(r for r, _, _ in table[:rank])
+    return row0, sum(r for r, _, _ in table)
+
+
 class Comm:
     """NCCL communicator for sat_sharded, bootstrapped over a torch process group: rank 0 creates the
     128-byte NCCL id, the group broadcasts it, every rank calls sat_comm_init collectively."""
@@ -147,18 +184,10 @@ class Comm:
     def __init__(self, group=None):
         import torch.distributed as dist
 
-        torch = _torch()
         self.group = group
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
-        buf = ctypes.create_string_buffer(128)
-        if self.rank == 0:
-            check(_lib.lib().sat_comm_get_unique_id(buf), "sat_comm_get_unique_id")
-        backend = dist.get_backend(group)
-        dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
-        t = torch.frombuffer(bytearray(buf.raw), dtype=torch.uint8).to(dev)
-        dist.broadcast(t, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
-        raw = bytes(t.cpu().tolist())
+        raw = broadcast_unique_id(group)
         self._h = ctypes.c_void_p()
         check(_lib.lib().sat_comm_init(ctypes.byref(self._h), raw, self.world, self.rank), "sat_comm_init")
 
@@ -174,11 +203,14 @@ class Comm:
             pass
 
 
-def sat_sharded(strip, out=None, *, comm: Comm, stream=None):
+def sat_sharded(strip, out=None, *, comm: Comm, stream=None, check_layout: bool = False):
     """Strip-partitioned SAT: this rank's horizontal strip in, this rank's strip of the global SAT out.
-    Collective over ``comm`` (call on every rank in the same order, equal column counts)."""
+    Collective over ``comm`` (call on every rank in the same order, equal column counts).  With
+    ``check_layout`` the ranks first verify the partition (strip_layout, one small collective)."""
     torch = _torch()
     rows, cols, pitch = _matrix(strip, "strip") if strip.shape[0] > 0 else (0, strip.shape[1], strip.shape[1])
+    if check_layout:
+        strip_layout(rows, cols, _dtype_code(strip), comm.group)
     if out is None:
         out = torch.empty_strided((rows, cols), (pitch, 1), dtype=strip.dtype, device=strip.device)
     with torch.cuda.device(strip.device):

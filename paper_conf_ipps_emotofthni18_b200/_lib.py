@@ -33,7 +33,8 @@ class SatPlan(ctypes.Structure):
     _fields_ = [
         ("tile_rows", ctypes.c_int32), ("tile_cols", ctypes.c_int32), ("tma", ctypes.c_int32),
         ("ctas", ctypes.c_int32), ("tiles", ctypes.c_int64), ("aux_bytes", ctypes.c_int64),
-        ("variant", ctypes.c_int32), ("order", ctypes.c_int32),
+        ("variant", ctypes.c_int32), ("order", ctypes.c_int32), ("family", ctypes.c_int32),
+        ("reserved", ctypes.c_int32),
     ]
 
 

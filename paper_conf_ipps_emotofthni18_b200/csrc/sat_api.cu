@@ -60,6 +60,7 @@ using PrepareFn = cudaError_t (*)(bool tma, bool carry, int* occupancy);
 
 struct Variant {
     int TR, TC, NW, STAGES;
+    int family;            // 1 = warp-specialised (sat_ws_kernel), 0 = classic (sat_tiles_kernel)
     size_t smem;           // dynamic shared memory bytes (same for int32 / fp32)
     LaunchFn launch[2];    // [dtype]
     PrepareFn prepare[2];  // [dtype]
@@ -74,6 +75,7 @@ template <int TR, int TC, int NW, int ST>
 struct Family<sat::TileCfg<TR, TC, NW, ST>> {
     using Cfg = sat::TileCfg<TR, TC, NW, ST>;
     static constexpr int threads = NW * 32;
+    static constexpr int family = 0;
     template <typename V>
     static constexpr size_t smem() { return sizeof(sat::Smem<V, Cfg>); }
     template <typename V, bool TMA, bool CARRY>
@@ -84,6 +86,7 @@ template <int TR, int NW, int ST, int NT>
 struct Family<sat::WsCfg<TR, NW, ST, NT>> {
     using Cfg = sat::WsCfg<TR, NW, ST, NT>;
     static constexpr int threads = Cfg::THREADS;
+    static constexpr int family = 1;
     template <typename V>
     static constexpr size_t smem() { return sizeof(sat::WsSmem<V, Cfg>); }
     template <typename V, bool TMA, bool CARRY>
@@ -122,6 +125,7 @@ Variant make_variant() {
     v.TC = Cfg::TC;
     v.NW = Cfg::NW;
     v.STAGES = Cfg::STAGES;
+    v.family = Family<Cfg>::family;
     v.smem = Family<Cfg>::template smem<uint32_t>();
     v.launch[SAT_INT32] = &launch_variant<uint32_t, Cfg>;
     v.launch[SAT_FLOAT32] = &launch_variant<float, Cfg>;
@@ -747,6 +751,8 @@ SAT_API sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t col
     plan->aux_bytes = pl.ntiles * (v.TR + v.TC + 1) * 8;
     plan->variant = pl.vi;
     plan->order = pl.order;
+    plan->family = v.family;
+    plan->reserved = 0;
     plan->ctas = 0;
     int dev = 0;
     if (cudaGetDevice(&dev) == cudaSuccess) {

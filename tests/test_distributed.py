@@ -1,0 +1,118 @@
+"""Multi-process host logic of the strip-partitioned path (BASELINE.json configs[4]) on CPU with the
+gloo backend, world size 2 and 3: the NCCL id bootstrap, the strip partition check, and the carry
+exchange protocol (which ranks' column sums enter a rank's carry, in which order) replayed with the
+oracle's arithmetic through real torch.distributed collectives.  The device kernels of the same
+path are covered by tests/test_gpu_parity.py (fake exchange on one GPU, and a 1-rank NCCL run)."""
+import os
+import socket
+import traceback
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+import torch.distributed as dist  # noqa: E402
+import torch.multiprocessing as mp  # noqa: E402
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _run(world, fn, *args):
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_entry, args=(r, world, port, fn, args, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    results = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    errs = [r for r in results if r[1] is not None]
+    assert not errs, errs[0][1]
+    return {r[0]: r[2] for r in results}
+
+
+def _entry(rank, world, port, fn, args, q):
+    try:
+        import sys
+        from pathlib import Path
+
+        root = str(Path(__file__).resolve().parent.parent)
+        sys.path.insert(0, root)
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        out = fn(rank, world, *args)
+        dist.barrier()
+        dist.destroy_process_group()
+        q.put((rank, None, out))
+    except Exception:
+        q.put((rank, traceback.format_exc(), None))
+
+
+# ----------------------------------------------------------------------------------------- workers
+def _w_unique_id(rank, world):
+    import paper_conf_ipps_emotofthni18_b200 as sat
+
+    raw = sat.broadcast_unique_id()
+    assert len(raw) == 128
+    gathered = [None] * world
+    dist.all_gather_object(gathered, raw)
+    assert all(g == gathered[0] for g in gathered)
+    return raw.hex()
+
+
+def _w_layout(rank, world, heights, cols_per_rank):
+    import paper_conf_ipps_emotofthni18_b200 as sat
+
+    try:
+        row0, total = sat.strip_layout(heights[rank], cols_per_rank[rank], sat.SAT_INT32)
+        return ("ok", row0, total)
+    except ValueError as e:
+        return ("mismatch", str(e))
+
+
+def _w_carry_exchange(rank, world, rows, cols, seed):
+    """The exchange of sat_compute_sharded with oracle arithmetic: colsum of my strip -> all_gather ->
+    C_r = sum_{g<r} colsum_g (ascending g) -> carry = row-wise prefix of C_r; then my strip of the SAT
+    is carry + SAT(strip).  Checked against the oracle SAT of the whole matrix."""
+    import oracle
+    import paper_conf_ipps_emotofthni18_b200 as sat
+    import satgen
+
+    row0, n = sat.strip_bounds(rows, world, rank)
+    strip = satgen.gen_host(n, cols, seed, "u32", row0=row0)
+    r0_chk, total = sat.strip_layout(n, cols, sat.SAT_INT32)
+    assert (r0_chk, total) == (row0, rows)
+    colsum = oracle.strip_carry_u32(strip, cols)  # column sums of my strip (mod 2^32)
+    gathered = [torch.zeros(cols, dtype=torch.int64) for _ in range(world)]
+    dist.all_gather(gathered, torch.from_numpy(colsum.astype(np.int64)))
+    C = np.zeros(cols, dtype=np.uint64)
+    for g in range(rank):  # ascending rank order (reading R12)
+        C = (C + gathered[g].numpy().astype(np.uint64)) % (1 << 32)
+    carry = oracle.row_prefix_u32(C.astype(np.uint32)[None, :])[0]
+    mine = (oracle.sat_u32(strip).astype(np.uint64) + carry.astype(np.uint64)[None, :]) % (1 << 32)
+    full = oracle.sat_u32(satgen.gen_host(rows, cols, seed, "u32"))
+    assert (mine.astype(np.uint32) == full[row0:row0 + n]).all()
+    return int(mine.astype(np.uint64).sum() % (1 << 32)) if n else 0
+
+
+# ----------------------------------------------------------------------------------------- tests
+def test_unique_id_broadcast_gloo():
+    ids = _run(2, _w_unique_id)
+    assert ids[0] == ids[1]
+
+
+def test_strip_layout_consistent_and_mismatch():
+    res = _run(3, _w_layout, [5, 7, 0], [11, 11, 11])
+    assert res[0] == ("ok", 0, 12) and res[1] == ("ok", 5, 12) and res[2] == ("ok", 12, 12)
+    bad = _run(2, _w_layout, [4, 4], [11, 12])
+    assert all(r[0] == "mismatch" for r in bad.values())
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_carry_exchange_protocol_gloo(world):
+    _run(world, _w_carry_exchange, 61, 45, 1447 + world)
