@@ -24,7 +24,7 @@ STATUS_NAMES = {
 EXPORTS = (
     "sat_compute_i32", "sat_compute_f32", "sat_compute", "sat_compute_host", "sat_strip_colsum",
     "sat_carry_prefix", "sat_comm_get_unique_id", "sat_comm_init", "sat_comm_destroy", "sat_compute_sharded",
-    "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order", "sat_debug_stats",
+    "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order", "sat_debug_stats", "sat_debug_trace",
     "sat_release_workspaces", "sat_status_string", "sat_last_error_detail", "sat_version",
 )
 
@@ -66,6 +66,7 @@ def _declare(lib):
         "sat_variant_info": [_int, ctypes.POINTER(_i32), ctypes.POINTER(_i32)],
         "sat_debug_tile_order": [_i64, _i64, _int, _vp, _vp],
         "sat_debug_stats": [_vp, _int, ctypes.POINTER(_int), ctypes.POINTER(_int)],
+        "sat_debug_trace": [_vp, _i64, ctypes.POINTER(_i64)],
         "sat_release_workspaces": [],
         "sat_status_string": [_int],
         "sat_last_error_detail": [],

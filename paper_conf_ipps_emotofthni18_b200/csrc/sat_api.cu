@@ -82,9 +82,9 @@ struct Family<sat::TileCfg<TR, TC, NW, ST>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_tiles_kernel<V, Cfg, TMA, CARRY>); }
 };
 
-template <int TR, int NW, int ST, int NT>
-struct Family<sat::WsCfg<TR, NW, ST, NT>> {
-    using Cfg = sat::WsCfg<TR, NW, ST, NT>;
+template <int TR, int NW, int ST, int NT, int NQ>
+struct Family<sat::WsCfg<TR, NW, ST, NT, NQ>> {
+    using Cfg = sat::WsCfg<TR, NW, ST, NT, NQ>;
     static constexpr int threads = Cfg::THREADS;
     static constexpr int family = 1;
     template <typename V>
@@ -136,10 +136,10 @@ Variant make_variant() {
 
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
-        make_variant<sat::WsCfg<128, 16, 3, 2>>(),  // 0: warp-specialised, 64 KiB tiles, 3 stages
-        make_variant<sat::WsCfg<128, 16, 3, 1>>(),  // 1: ... one tile in flight per walker
-        make_variant<sat::WsCfg<64, 16, 6, 2>>(),   // 2: warp-specialised, 32 KiB tiles, 6 stages
-        make_variant<sat::WsCfg<64, 8, 6, 2>>(),    // 3: ... 8 compute warps
+        make_variant<sat::WsCfg<128, 16, 3, 1, 5>>(),  // 0: warp-specialised, 64 KiB tiles, 3 stages, 5-tile ring
+        make_variant<sat::WsCfg<128, 16, 3, 1, 3>>(),  // 1: ... tickets only as stages free up
+        make_variant<sat::WsCfg<128, 16, 3, 2, 6>>(),  // 2: ... 6-tile ring, two tiles per walker
+        make_variant<sat::WsCfg<64, 16, 6, 2, 8>>(),   // 3: warp-specialised, 32 KiB tiles, 6 stages, 8-tile ring
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 4: classic, 32 KiB tiles, 2 stages
         make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 5: classic, 64 KiB tiles, 512 threads
     };
@@ -156,7 +156,7 @@ int g_max_ctas = 0;
 int auto_variant(int64_t rows, int64_t cols) {
     (void)cols;
     (void)rows;
-    return 1;  // best measured at 32K x 32K (tools/sweep_variants.py)
+    return 0;  // best measured at 32K x 32K (tools/sweep_variants.py)
 }
 
 // ------------------------------------------------------------------ device info caches
@@ -202,8 +202,10 @@ struct Workspace {
     uint64_t* slots = nullptr;
     size_t slot_words = 0;
     uint64_t calls = 0;
-    long long* stats = nullptr;  // SAT_STATS builds: [ctas][kNumStats] of the last launch
+    long long* stats = nullptr;  // SAT_STATS builds: [ctas][kNumStats] of the last launch, then the trace
     int stats_ctas = 0;
+    size_t stats_words = 0;
+    int64_t trace_tiles = 0;
     void* scratch = nullptr;  // colsum partials etc.
     size_t scratch_bytes = 0;
 };
@@ -413,14 +415,21 @@ sat_status_t compute_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ro
     p.ctrl = w->ctrl;
     p.carry = static_cast<const uint32_t*>(carry);
     p.stats = nullptr;
+    p.trace = nullptr;
 #if SAT_STATS
-    if (w->stats_ctas < grid) {
-        if (w->stats) cudaFree(w->stats);
-        SAT_CUDA(cudaMalloc(&w->stats, static_cast<size_t>(grid) * sat::kNumStats * 8));
+    {
+        const size_t need = static_cast<size_t>(grid) * sat::kNumStats + 2 * static_cast<size_t>(pl.ntiles);
+        if (w->stats_words < need) {
+            if (w->stats) cudaFree(w->stats);
+            SAT_CUDA(cudaMalloc(&w->stats, need * 8));
+            w->stats_words = need;
+        }
+        w->stats_ctas = static_cast<int>(grid);
+        w->trace_tiles = pl.ntiles;
+        SAT_CUDA(cudaMemsetAsync(w->stats, 0, need * 8, st));
+        p.stats = w->stats;
+        p.trace = w->stats + static_cast<size_t>(grid) * sat::kNumStats;
     }
-    w->stats_ctas = static_cast<int>(grid);
-    SAT_CUDA(cudaMemsetAsync(w->stats, 0, static_cast<size_t>(grid) * sat::kNumStats * 8, st));
-    p.stats = w->stats;
     g_last_stats = w;
 #endif
     cudaError_t e = v.launch[dt](pl.tma, carry != nullptr, dim3(static_cast<unsigned>(grid)), st, mi, mo, &p);
@@ -825,6 +834,23 @@ SAT_API sat_status_t sat_debug_stats(int64_t* out, int max_ctas, int* n_ctas, in
     return SAT_OK;
 #else
     (void)out; (void)max_ctas; (void)n_ctas; (void)n_stats;
+    return fail(SAT_ERR_UNSUPPORTED, "libsat built without SAT_STATS");
+#endif
+}
+
+SAT_API sat_status_t sat_debug_trace(int64_t* out, int64_t max_tiles, int64_t* n_tiles) {
+#if SAT_STATS
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (!g_last_stats || !out || !n_tiles) return fail(SAT_ERR_INVALID_VALUE, "no trace");
+    Workspace* w = g_last_stats;
+    const int64_t n = w->trace_tiles < max_tiles ? w->trace_tiles : max_tiles;
+    SAT_CUDA(cudaStreamSynchronize(w->stream));
+    SAT_CUDA(cudaMemcpy(out, w->stats + static_cast<size_t>(w->stats_ctas) * sat::kNumStats,
+                        static_cast<size_t>(n) * 16, cudaMemcpyDeviceToHost));
+    *n_tiles = n;
+    return SAT_OK;
+#else
+    (void)out; (void)max_tiles; (void)n_tiles;
     return fail(SAT_ERR_UNSUPPORTED, "libsat built without SAT_STATS");
 #endif
 }

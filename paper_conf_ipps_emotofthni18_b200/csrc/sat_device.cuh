@@ -92,6 +92,23 @@ __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void*
                  : "memory");
 }
 
+// Same with an L2 eviction policy (evict_first for the streamed output, so it does not push the
+// look-back status words out of L2).
+__device__ __forceinline__ void tma_store_2d_hint(const CUtensorMap* map, const void* smem_src, int x, int y,
+                                                  uint64_t policy) {
+    asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%1, %2}], [%3], %4;" ::"l"(
+                     map),
+                 "r"(x), "r"(y), "r"(smem_addr(smem_src)), "l"(policy)
+                 : "memory");
+}
+
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 
 template <int N>
@@ -127,6 +144,47 @@ __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
 }
 __device__ __forceinline__ void ld_relaxed2(const uint64_t* p, uint64_t& a, uint64_t& b) {
     asm volatile("ld.relaxed.gpu.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+
+// Status-word accesses with an L2 evict_last policy: the words must survive in L2 between their
+// publication and their successors' look-backs while the matrix streams through.
+__device__ __forceinline__ void st_relaxed_p(uint64_t* p, uint64_t a, uint64_t pol) {
+    asm volatile("st.relaxed.gpu.global.L2::cache_hint.b64 [%0], %1, %2;" ::"l"(p), "l"(a), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void st_relaxed2_p(uint64_t* p, uint64_t a, uint64_t b, uint64_t pol) {
+    asm volatile("st.relaxed.gpu.global.L2::cache_hint.v2.b64 [%0], {%1, %2}, %3;" ::"l"(p), "l"(a), "l"(b), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ uint64_t ld_relaxed_p(const uint64_t* p, uint64_t pol) {
+    uint64_t a;
+    asm volatile("ld.relaxed.gpu.global.L2::cache_hint.b64 %0, [%1], %2;" : "=l"(a) : "l"(p), "l"(pol) : "memory");
+    return a;
+}
+__device__ __forceinline__ void ld_relaxed2_p(const uint64_t* p, uint64_t& a, uint64_t& b, uint64_t pol) {
+    asm volatile("ld.relaxed.gpu.global.L2::cache_hint.v2.b64 {%0, %1}, [%2], %3;"
+                 : "=l"(a), "=l"(b)
+                 : "l"(p), "l"(pol)
+                 : "memory");
+}
+
+template <int E>
+__device__ __forceinline__ void st_words_p(uint64_t* p, const uint64_t (&w)[E], uint64_t pol) {
+    if constexpr (E == 1) {
+        st_relaxed_p(p, w[0], pol);
+    } else {
+#pragma unroll
+        for (int e = 0; e < E; e += 2) st_relaxed2_p(p + e, w[e], w[e + 1], pol);
+    }
+}
+
+template <int E>
+__device__ __forceinline__ void ld_words_p(const uint64_t* p, uint64_t (&w)[E], uint64_t pol) {
+    if constexpr (E == 1) {
+        w[0] = ld_relaxed_p(p, pol);
+    } else {
+#pragma unroll
+        for (int e = 0; e < E; e += 2) ld_relaxed2_p(p + e, w[e], w[e + 1], pol);
+    }
 }
 
 template <int E>

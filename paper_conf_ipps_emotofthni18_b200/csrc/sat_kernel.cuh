@@ -38,7 +38,7 @@ constexpr uint32_t kEpochMax = (1u << 30) - 1u;
 #ifndef SAT_STATS
 #define SAT_STATS 0
 #endif
-constexpr int kNumStats = 20;
+constexpr int kNumStats = 24;
 enum StatSlot {
     kStTiles = 0, kStLoop, kStTicket, kStFullWait, kStCompute, kStRowLb, kStRowSteps, kStRowSpins, kStColLb,
     kStColSteps, kStColSpins, kStDiagTry, kStDiagUnresolved, kStDiagLate, kStBar3Producer, kStStore,
@@ -73,6 +73,7 @@ struct KParams {
     Ctrl* ctrl;
     const V* carry;    // [cols] or nullptr
     long long* stats;  // [gridDim.x][kNumStats] (SAT_STATS builds only) or nullptr
+    long long* trace;  // [ntiles][2]: acquisition / store-issue globaltimer ns (SAT_STATS builds only)
 };
 
 __device__ __forceinline__ uint64_t pack(uint32_t epoch, uint32_t kind, uint32_t bits) {

@@ -34,7 +34,8 @@ namespace sat {
 // Stats builds (-DSAT_STATS=1): per-CTA counters in shared memory, role-tagged slots.
 enum WsStat {
     kWsTiles = 0, kWsFullWait, kWsLocal, kWsWalkWait, kWsFinish, kWsRowRounds, kWsColRounds,
-    kWsStResultWait, kWsStStore, kWsLdIssue, kWsLdEmptyWait, kWsBandBar, kWsRowTiles, kWsColTiles
+    kWsStResultWait, kWsStStore, kWsLdIssue, kWsLdEmptyWait, kWsBandBar, kWsRowTiles, kWsColTiles,
+    kWsRowRoundCyc, kWsColRoundCyc, kWsRowResolve, kWsColResolve, kWsRowIdle, kWsColIdle, kWsRowLat, kWsColLat
 };
 #if SAT_STATS
 __shared__ unsigned long long ws_stats[kNumStats];
@@ -42,6 +43,12 @@ __shared__ unsigned long long ws_stats[kNumStats];
 #else
 #define WS_ST(k, v) (void)0
 #endif
+
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
@@ -77,9 +84,10 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-template <int TR_, int NW_, int STAGES_, int NT_>
+template <int TR_, int NW_, int STAGES_, int NT_, int NQ_>
 struct WsCfg {
     static constexpr int TR = TR_, TC = 128, NW = NW_, STAGES = STAGES_;
+    static constexpr int NQ = NQ_;        // tile ring: tiles acquired ahead of their data stage
     static constexpr int NT = NT_;        // tiles in flight per walker
     static constexpr int RPW = TR / NW;   // rows per compute-warp band
     static constexpr int ER = TR / 32;    // row-vector elements per walker lane
@@ -90,23 +98,27 @@ struct WsCfg {
     static_assert(TR % NW == 0 && TR % 32 == 0, "tile shape");
     static_assert(RPW % 2 == 0, "row slots are published in pairs");
     static_assert(ER == 1 || ER % 2 == 0, "row vector split");
-    static_assert(STAGES >= 2 && STAGES <= 8 && NT >= 1, "ring");
+    static_assert(STAGES >= 2 && STAGES <= 8 && NT >= 1 && NQ >= STAGES && NQ <= 16, "rings");
 };
 
+// Two rings: the data stages (tile k's pixels live in stage k % STAGES) and the tile ring (tile k's
+// id, carries and hand-off barriers live in slot k % NQ).  Tiles are acquired up to NQ ahead of the
+// storer, i.e. before a data stage is free, so their look-backs start earlier.
 template <typename V, typename Cfg>
 struct WsSmem {
     alignas(1024) V stage[Cfg::STAGES][Cfg::TR * Cfg::TC];
     alignas(16) V band[2][Cfg::NW][Cfg::TC];
-    alignas(16) V rp[Cfg::STAGES][Cfg::TR];  // row carry    prefix_i GRS(I,J-1)
-    alignas(16) V cp[Cfg::STAGES][Cfg::TC];  // column carry prefix_j GCS(I-1,J)
-    V corner[Cfg::STAGES];                   // GS(I-1,J-1)
-    alignas(8) uint64_t acq[Cfg::STAGES];
-    uint64_t full[Cfg::STAGES];
-    uint64_t rowwalk[Cfg::STAGES];
-    uint64_t colwalk[Cfg::STAGES];
+    alignas(16) V rp[Cfg::NQ][Cfg::TR];  // row carry    prefix_i GRS(I,J-1)
+    alignas(16) V cp[Cfg::NQ][Cfg::TC];  // column carry prefix_j GCS(I-1,J)
+    V corner[Cfg::NQ];                   // GS(I-1,J-1)
+    alignas(8) uint64_t acq[Cfg::NQ];    // tile id written (tile ring)
+    uint64_t rowwalk[Cfg::NQ];
+    uint64_t colwalk[Cfg::NQ];
+    uint64_t tfree[Cfg::NQ];             // tile slot released by the storer
+    uint64_t full[Cfg::STAGES];          // data ring
     uint64_t result[Cfg::STAGES];
     uint64_t empty[Cfg::STAGES];
-    alignas(16) TileInfo info[Cfg::STAGES];
+    alignas(16) TileInfo info[Cfg::NQ];
     uint32_t epoch;
     int end_n;  // index of the end marker once the loader has drawn an invalid ticket, else INT_MAX
 };
@@ -163,7 +175,7 @@ __device__ __forceinline__ bool lb_consume(uint32_t& pending, int& pos, V (&acc)
 
 template <typename V, typename Cfg, bool ROW>
 __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
-    constexpr int TR = Cfg::TR, TC = Cfg::TC, STAGES = Cfg::STAGES;
+    constexpr int TR = Cfg::TR, TC = Cfg::TC;
     constexpr int E = ROW ? Cfg::ER : Cfg::EC;
     constexpr int NT = Cfg::NT;
     struct Walk {
@@ -172,13 +184,16 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
         V acc[E];
         V dacc;
         int dbase, ddone;
+        long long t_acq;
     };
     Walk wk[NT];
 #pragma unroll
     for (int w = 0; w < NT; ++w) wk[w].active = 0;
-    Slot<STAGES> next;
+    Slot<Cfg::NQ> next;
     bool ended = false;
     int steps = 0;
+    const uint64_t pol = policy_evict_last();
+    constexpr int DW = 4;  // diagonal predecessors polled per round (the first is almost always inclusive)
     while (true) {
         // ---- take newly acquired tiles into free walk slots (block only when nothing is in flight)
 #pragma unroll
@@ -213,6 +228,9 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
             x.dacc = V(0);
             x.dbase = 1;
             x.ddone = ROW ? (ti.I == 0 || ti.J == 0) : 1;
+#if SAT_STATS
+            x.t_acq = clock64();
+#endif
             next.next();
         }
         bool any = false;
@@ -232,18 +250,40 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
             if (x.pend) {
                 if (ROW) {
                     const long long base = static_cast<long long>(x.I) * p.C;
-                    ld_words<E>(p.row_slots + (base + x.pos) * TR + lane * E, w0[w]);
-                    if (x.pos >= 1) ld_words<E>(p.row_slots + (base + x.pos - 1) * TR + lane * E, w1[w]);
+                    ld_words_p<E>(p.row_slots + (base + x.pos) * TR + lane * E, w0[w], pol);
+                    if (x.pos >= 1) ld_words_p<E>(p.row_slots + (base + x.pos - 1) * TR + lane * E, w1[w], pol);
                 } else {
-                    ld_words<E>(p.col_slots + (static_cast<long long>(x.pos) * p.C + x.J) * TC + lane * E, w0[w]);
+                    ld_words_p<E>(p.col_slots + (static_cast<long long>(x.pos) * p.C + x.J) * TC + lane * E, w0[w],
+                                  pol);
                     if (x.pos >= 1)
-                        ld_words<E>(p.col_slots + (static_cast<long long>(x.pos - 1) * p.C + x.J) * TC + lane * E,
-                                    w1[w]);
+                        ld_words_p<E>(p.col_slots + (static_cast<long long>(x.pos - 1) * p.C + x.J) * TC + lane * E,
+                                      w1[w], pol);
                 }
             }
-            if (ROW && !x.ddone) wd[w] = diag_word(p.corner_slots, x.I, x.J, p.C, x.dbase + lane);
+            if (ROW && !x.ddone && lane < DW) {
+                const int kk = x.dbase + lane;
+                if (x.I - kk >= 0 && x.J - kk >= 0)
+                    wd[w] = ld_relaxed_p(p.corner_slots + static_cast<long long>(x.I - kk) * p.C + (x.J - kk), pol);
+            }
         }
         ++steps;
+        SAT_CLK(r0);
+#if SAT_STATS
+        {   // stats only: wait for the round's loads to measure their latency apart from processing
+            uint64_t sink = 0;
+#pragma unroll
+            for (int w = 0; w < NT; ++w) {
+                if (wk[w].active && wk[w].pend) {
+#pragma unroll
+                    for (int e = 0; e < E; ++e) sink ^= w0[w][e];
+                }
+                sink ^= wd[w];
+            }
+            if (sink == 0x123456789abcdefull) wk[0].J = -7;  // never true; forces the loads to land
+            SAT_CLK(rl);
+            if (lane == 0) WS_ST(ROW ? kWsRowLat : kWsColLat, rl - r0);
+        }
+#endif
         // ---- ... then consume them
         bool progress = false;
 #pragma unroll
@@ -253,17 +293,20 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
             if (x.pend) progress |= lb_consume<V, E>(x.pend, x.pos, x.acc, w0[w], w1[w], x.pos >= 1, epoch);
             if (ROW && !x.ddone) {
                 // Step 3.2: GS(I-1,J-1) = GS(I-k,J-k) + sum of GLS of the tiles between
+                // window of DW lanes; the grid-edge tile of a diagonal is always inclusive
                 const int kk = x.dbase + lane;
-                const bool inrange = (x.I - kk >= 0) && (x.J - kk >= 0);
+                const bool inrange = lane < DW && (x.I - kk >= 0) && (x.J - kk >= 0);
                 const bool ready = !inrange || word_ready(wd[w], epoch);
                 const unsigned incl = __ballot_sync(kFull, inrange && ready && word_kind(wd[w]) == kIncl);
                 const unsigned notready = __ballot_sync(kFull, !ready);
-                const int f = incl ? (__ffs(incl) - 1) : 32;
-                const unsigned need = (f >= 31) ? kFull : ((2u << f) - 1u);
+                const int f = incl ? (__ffs(incl) - 1) : DW;
+                const unsigned need = (2u << (f < DW ? f : DW - 1)) - 1u;
                 if (!(notready & need)) {
-                    const V val = (inrange && lane <= f) ? from_bits<V>(static_cast<uint32_t>(wd[w])) : V(0);
-                    x.dacc = x.dacc + warp_sum(val);
-                    if (f < 32) x.ddone = 1; else x.dbase += 32;
+                    V val = (inrange && lane <= f) ? from_bits<V>(static_cast<uint32_t>(wd[w])) : V(0);
+#pragma unroll
+                    for (int d = DW / 2; d >= 1; d >>= 1) val = val + __shfl_xor_sync(kFull, val, d);
+                    x.dacc = x.dacc + __shfl_sync(kFull, val, 0);
+                    if (f < DW) x.ddone = 1; else x.dbase += DW;
                     progress = true;
                 }
             }
@@ -280,12 +323,20 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
                 if (lane == 0) {
                     mbar_arrive(ROW ? &sm.rowwalk[x.s] : &sm.colwalk[x.s]);
                     WS_ST(ROW ? kWsRowTiles : kWsColTiles, 1);
+#if SAT_STATS
+                    WS_ST(ROW ? kWsRowResolve : kWsColResolve, clock64() - x.t_acq);
+#endif
                 }
                 x.active = 0;
                 progress = true;
             }
         }
-        if (!__any_sync(kFull, progress)) __nanosleep(64);
+        SAT_CLK(r1);
+        if (lane == 0) WS_ST(ROW ? kWsRowRoundCyc : kWsColRoundCyc, r1 - r0);
+        if (!__any_sync(kFull, progress)) {
+            if (lane == 0) WS_ST(ROW ? kWsRowIdle : kWsColIdle, 1);
+            __nanosleep(64);
+        }
     }
     if (lane == 0) WS_ST(ROW ? kWsRowRounds : kWsColRounds, steps);
 }
@@ -294,8 +345,8 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
 // at the end marker.
 template <typename V, typename Cfg, bool TMA>
 __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p, V (&v)[Cfg::RPW][4],
-                                         const Slot<Cfg::STAGES>& sl, int& I, int& J, uint32_t epoch, int warp,
-                                         int lane) {
+                                         const Slot<Cfg::STAGES>& sl, const Slot<Cfg::NQ>& tq, int& I, int& J,
+                                         uint32_t epoch, int warp, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
     const int s = sl.s;
     const int row0 = warp * RPW, col0 = lane * 4;
@@ -303,7 +354,7 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
     mbar_wait(&sm.full[s], sl.ph);
     SAT_CLK(c1);
     if (warp == 0 && lane == 0) { WS_ST(kWsFullWait, c1 - c0); WS_ST(kWsTiles, 1); }
-    const TileInfo ti = sm.info[s];
+    const TileInfo ti = sm.info[tq.s];
     if (ti.t >= p.ntiles) return false;
     I = ti.I;
     J = ti.J;
@@ -389,18 +440,20 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
     // ---- Steps 2.A.1 / 2.B.1: local aggregates (prefix form) from the owning lanes: the last column
     //      (lane 31 of every warp) and the bottom row (last warp).  Edge tiles publish inclusive at
     //      once: their carry is zero.
+    const uint64_t pol = policy_evict_last();
     if (lane == 31) {
         uint64_t* rs = p.row_slots + tidx * TR + row0;
         const uint32_t kind = (J == 0) ? kIncl : kLocal;
 #pragma unroll
         for (int r = 0; r < RPW; r += 2)
-            st_relaxed2(rs + r, pack(epoch, kind, to_bits(v[r][3])), pack(epoch, kind, to_bits(v[r + 1][3])));
+            st_relaxed2_p(rs + r, pack(epoch, kind, to_bits(v[r][3])), pack(epoch, kind, to_bits(v[r + 1][3])), pol);
     }
     if (warp == NW - 1) {
         uint64_t* cs = p.col_slots + tidx * TC + col0;
         const uint32_t kind = (I == 0) ? kIncl : kLocal;
-        st_relaxed2(cs, pack(epoch, kind, to_bits(v[RPW - 1][0])), pack(epoch, kind, to_bits(v[RPW - 1][1])));
-        st_relaxed2(cs + 2, pack(epoch, kind, to_bits(v[RPW - 1][2])), pack(epoch, kind, to_bits(v[RPW - 1][3])));
+        st_relaxed2_p(cs, pack(epoch, kind, to_bits(v[RPW - 1][0])), pack(epoch, kind, to_bits(v[RPW - 1][1])), pol);
+        st_relaxed2_p(cs + 2, pack(epoch, kind, to_bits(v[RPW - 1][2])), pack(epoch, kind, to_bits(v[RPW - 1][3])),
+                      pol);
     }
     SAT_CLK(c2);
     if (warp == 0 && lane == 0) WS_ST(kWsLocal, c2 - c1);
@@ -410,45 +463,47 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
 // Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 and Step 4 for the tile in stage sl.s whose local SAT is in `v`.
 template <typename V, typename Cfg, bool TMA, bool CARRY>
 __device__ __forceinline__ void ws_finish(WsSmem<V, Cfg>& sm, const KParams<V>& p, V (&v)[Cfg::RPW][4],
-                                          const Slot<Cfg::STAGES>& sl, int I, int J, uint32_t epoch, int warp,
-                                          int lane) {
+                                          const Slot<Cfg::STAGES>& sl, const Slot<Cfg::NQ>& tq, int I, int J,
+                                          uint32_t epoch, int warp, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
-    const int s = sl.s;
+    const int s = sl.s, q = tq.s;
     const int row0 = warp * RPW, col0 = lane * 4;
     const long long tidx = static_cast<long long>(I) * p.C + J;
+    const uint64_t pol = policy_evict_last();
     SAT_CLK(c0);
-    mbar_wait(&sm.rowwalk[s], sl.ph);
-    mbar_wait(&sm.colwalk[s], sl.ph);
+    mbar_wait(&sm.rowwalk[q], tq.ph);
+    mbar_wait(&sm.colwalk[q], tq.ph);
     SAT_CLK(c1);
     if (warp == 0 && lane == 0) WS_ST(kWsWalkWait, c1 - c0);
     V rt[RPW];
 #pragma unroll
-    for (int r = 0; r < RPW; ++r) rt[r] = sm.rp[s][row0 + r];
+    for (int r = 0; r < RPW; ++r) rt[r] = sm.rp[q][row0 + r];
     V cpv[4];
     {
-        const uint4 q = *reinterpret_cast<const uint4*>(&sm.cp[s][col0]);
-        cpv[0] = from_bits<V>(q.x); cpv[1] = from_bits<V>(q.y); cpv[2] = from_bits<V>(q.z); cpv[3] = from_bits<V>(q.w);
+        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[q][col0]);
+        cpv[0] = from_bits<V>(c4.x); cpv[1] = from_bits<V>(c4.y); cpv[2] = from_bits<V>(c4.z);
+        cpv[3] = from_bits<V>(c4.w);
     }
-    const V corner = sm.corner[s];
+    const V corner = sm.corner[q];
     // inclusive aggregates, from the lanes that hold the local ones
     if (lane == 31 && J > 0) {
         uint64_t* rs = p.row_slots + tidx * TR + row0;
 #pragma unroll
         for (int r = 0; r < RPW; r += 2)
-            st_relaxed2(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + rt[r])),
-                        pack(epoch, kIncl, to_bits(v[r + 1][3] + rt[r + 1])));
+            st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + rt[r])),
+                          pack(epoch, kIncl, to_bits(v[r + 1][3] + rt[r + 1])), pol);
     }
     if (warp == NW - 1) {
         if (I > 0) {
             uint64_t* cs = p.col_slots + tidx * TC + col0;
-            st_relaxed2(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + cpv[0])),
-                        pack(epoch, kIncl, to_bits(v[RPW - 1][1] + cpv[1])));
-            st_relaxed2(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + cpv[2])),
-                        pack(epoch, kIncl, to_bits(v[RPW - 1][3] + cpv[3])));
+            st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + cpv[0])),
+                          pack(epoch, kIncl, to_bits(v[RPW - 1][1] + cpv[1])), pol);
+            st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + cpv[2])),
+                          pack(epoch, kIncl, to_bits(v[RPW - 1][3] + cpv[3])), pol);
         }
         if (lane == 31) {  // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
             const V gls = v[RPW - 1][3] + rt[RPW - 1] + cpv[3];
-            st_relaxed(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(corner + gls)));
+            st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(corner + gls)), pol);
         }
     }
     // GSAT(I,J) = localSAT + rp[i] + cp[j] + corner (+ carry[j])
@@ -508,11 +563,15 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         sm.epoch = *reinterpret_cast<volatile unsigned int*>(&p.ctrl->epoch);
         sm.end_n = 0x7fffffff;
 #pragma unroll
+        for (int q = 0; q < Cfg::NQ; ++q) {
+            mbar_init(&sm.acq[q], 1);
+            mbar_init(&sm.rowwalk[q], 1);
+            mbar_init(&sm.colwalk[q], 1);
+            mbar_init(&sm.tfree[q], 1);
+        }
+#pragma unroll
         for (int s = 0; s < STAGES; ++s) {
-            mbar_init(&sm.acq[s], 1);
             mbar_init(&sm.full[s], 1);
-            mbar_init(&sm.rowwalk[s], 1);
-            mbar_init(&sm.colwalk[s], 1);
             mbar_init(&sm.result[s], NW);
             mbar_init(&sm.empty[s], 1);
         }
@@ -524,10 +583,11 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
     if (warp < NW) {
         // ================================================================ compute warps
         V v[RPW][4];
-        for (Slot<STAGES> sl;; sl.next()) {
+        Slot<STAGES> sl;
+        for (Slot<Cfg::NQ> tq;; tq.next(), sl.next()) {
             int I, J;
-            if (!ws_local<V, Cfg, TMA>(sm, p, v, sl, I, J, epoch, warp, lane)) break;
-            ws_finish<V, Cfg, TMA, CARRY>(sm, p, v, sl, I, J, epoch, warp, lane);
+            if (!ws_local<V, Cfg, TMA>(sm, p, v, sl, tq, I, J, epoch, warp, lane)) break;
+            ws_finish<V, Cfg, TMA, CARRY>(sm, p, v, sl, tq, I, J, epoch, warp, lane);
         }
     } else if (warp == Cfg::ROW_WARP) {
         ws_walker<V, Cfg, true>(sm, p, epoch, lane);
@@ -537,11 +597,12 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         // ================================================================ storer (one lane)
         if (lane == 0) {
             if constexpr (TMA) prefetch_tensormap(&map_out);
-            int pending = -1;  // stage whose store was issued last and is not yet released
-            for (Slot<STAGES> sl;; sl.next()) {
+            const uint64_t spol = policy_evict_first();
+            Slot<STAGES> sl;
+            for (Slot<Cfg::NQ> tq;; tq.next(), sl.next()) {
                 const int s = sl.s;
-                mbar_wait(&sm.acq[s], sl.ph);
-                const TileInfo ti = sm.info[s];  // stays valid until this lane releases the stage
+                mbar_wait(&sm.acq[tq.s], tq.ph);
+                const TileInfo ti = sm.info[tq.s];  // stays valid until this lane releases the slot
                 if (ti.t >= p.ntiles) break;
                 SAT_CLK(u0);
                 mbar_wait(&sm.result[s], sl.ph);
@@ -551,28 +612,20 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 if constexpr (TMA) {
                     const bool ragged = (ti.J == p.C - 1) && (p.cols & 3) != 0;
                     if (!ragged) {
-                        tma_store_2d(&map_out, sm.stage[s], ti.J * TC, ti.I * TR);
+                        tma_store_2d_hint(&map_out, sm.stage[s], ti.J * TC, ti.I * TR, spol);
                         bulk_commit();
                         stored = true;
                     }
                 }
-                // two stores in flight: release the previous stage once its store has read smem
-                if (pending >= 0) {
-                    if (stored) bulk_wait_read<1>(); else bulk_wait_read<0>();
-                    mbar_arrive(&sm.empty[pending]);
-                }
-                if (stored) {
-                    pending = s;
-                } else {
-                    mbar_arrive(&sm.empty[s]);
-                    pending = -1;
-                }
+                mbar_arrive(&sm.tfree[tq.s]);  // the tile slot (id, carries) is no longer needed
+#if SAT_STATS
+                if (p.trace) p.trace[2LL * ti.t + 1] = static_cast<long long>(globaltimer_ns());
+#endif
+                // release the stage as soon as its store has read the shared memory
+                if (stored) bulk_wait_read<0>();
+                mbar_arrive(&sm.empty[s]);
                 SAT_CLK(u2);
                 WS_ST(kWsStStore, u2 - u1);
-            }
-            if (pending >= 0) {
-                bulk_wait_read<0>();
-                mbar_arrive(&sm.empty[pending]);
             }
             if constexpr (TMA) bulk_wait_all();
             __threadfence();
@@ -591,37 +644,50 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         }
     } else if (lane == 0) {
         // ================================================================ loader (one lane)
+        // Two independent cursors: tickets are drawn into the tile ring as soon as a tile slot is free
+        // (so the walkers start early); TMA loads follow into the data ring as stages free up.
         const uint64_t policy = TMA ? policy_evict_first() : 0ull;
         if constexpr (TMA) prefetch_tensormap(&map_in);
-        // the next ticket is drawn right after a load is issued, so its L2 round trip overlaps the
-        // wait for a free stage (a CTA holds at most STAGES+1 tiles)
-        unsigned int ticket = atomicAdd(&p.ctrl->counter, 1u);
-        for (Slot<STAGES> sl;; sl.next()) {
-            const int s = sl.s;
-            if (sl.k >= STAGES) {  // wait until the store of the stage's previous tile has read it
-                SAT_CLK(e0);
-                mbar_wait(&sm.empty[s], sl.ph ^ 1u);
-                SAT_CLK(e1);
-                WS_ST(kWsLdEmptyWait, e1 - e0);
+        Slot<Cfg::NQ> ta, tl;  // acquisition cursor; load cursor (tile ring)
+        Slot<STAGES> sl;       // load cursor (data ring)
+        bool acq_done = false;
+        while (true) {
+            bool progress = false;
+            if (!acq_done && (ta.k < Cfg::NQ || mbar_test(&sm.tfree[ta.s], ta.ph ^ 1u))) {
+                SAT_CLK(t0);
+                const int t = static_cast<int>(atomicAdd(&p.ctrl->counter, 1u));
+                const bool valid = t < p.ntiles;
+                TileInfo ti{t, 0, 0, 0};
+                if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
+                sm.info[ta.s] = ti;
+                if (!valid) {
+                    *reinterpret_cast<volatile int*>(&sm.end_n) = ta.k;
+                    acq_done = true;
+                }
+                mbar_arrive(&sm.acq[ta.s]);
+#if SAT_STATS
+                if (p.trace && valid) p.trace[2LL * t] = static_cast<long long>(globaltimer_ns());
+#endif
+                ta.next();
+                progress = true;
+                SAT_CLK(t1);
+                WS_ST(kWsLdIssue, t1 - t0);
             }
-            SAT_CLK(t0);
-            const int t = static_cast<int>(ticket);
-            const bool valid = t < p.ntiles;
-            TileInfo ti{t, 0, 0, 0};
-            if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
-            sm.info[s] = ti;
-            if (!valid) *reinterpret_cast<volatile int*>(&sm.end_n) = sl.k;
-            mbar_arrive(&sm.acq[s]);
-            if (TMA && valid) {
-                mbar_arrive_expect_tx(&sm.full[s], kTileBytes);
-                tma_load_2d(sm.stage[s], &map_in, &sm.full[s], ti.J * TC, ti.I * TR, policy);
-            } else {
-                mbar_arrive(&sm.full[s]);  // generic path (data read from global) or end marker
+            if (tl.k < ta.k && (sl.k < STAGES || mbar_test(&sm.empty[sl.s], sl.ph ^ 1u))) {
+                const TileInfo ti = sm.info[tl.s];
+                const bool valid = ti.t < p.ntiles;
+                if (TMA && valid) {
+                    mbar_arrive_expect_tx(&sm.full[sl.s], kTileBytes);
+                    tma_load_2d(sm.stage[sl.s], &map_in, &sm.full[sl.s], ti.J * TC, ti.I * TR, policy);
+                } else {
+                    mbar_arrive(&sm.full[sl.s]);  // generic path (data read from global) or end marker
+                }
+                tl.next();
+                sl.next();
+                progress = true;
+                if (!valid) break;
             }
-            if (valid) ticket = atomicAdd(&p.ctrl->counter, 1u);
-            SAT_CLK(t1);
-            WS_ST(kWsLdIssue, t1 - t0);
-            if (!valid) break;
+            if (!progress) __nanosleep(32);
         }
     }
 }

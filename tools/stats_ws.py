@@ -19,7 +19,8 @@ import satgen  # noqa: E402
 
 NAMES = ["tiles", "c_full_wait", "c_local", "c_walk_wait", "c_finish", "row_rounds", "col_rounds",
          "st_result_wait", "st_store", "ld_issue", "ld_empty_wait", "c_bandbar", "row_tiles", "col_tiles",
-         "x14", "x15", "x16", "x17", "x18", "x19"]
+         "row_round_cyc", "col_round_cyc", "row_resolve", "col_resolve", "row_idle_rounds", "col_idle_rounds",
+         "row_load_lat", "col_load_lat", "x22", "x23"]
 ap = argparse.ArgumentParser()
 ap.add_argument("--n", type=int, default=32768)
 ap.add_argument("--variants", default="0,1")
@@ -39,11 +40,11 @@ for v in [int(s) for s in a.variants.split(",")]:
     sat.sat(x, out=y)
     e1.record()
     torch.cuda.synchronize()
-    buf = np.zeros((4096, 20), dtype=np.int64)
+    buf = np.zeros((4096, 24), dtype=np.int64)
     nc, ns = ctypes.c_int(), ctypes.c_int()
     _lib.check(_lib.lib().sat_debug_stats(buf.ctypes.data, 4096, ctypes.byref(nc), ctypes.byref(ns)), "stats")
     st = buf[: nc.value]
     tiles = st[:, 0].sum()
     print(json.dumps({"variant": v, "ms": round(e0.elapsed_time(e1), 4), "ctas": int(nc.value), "tiles": int(tiles),
-                      "per_tile": {NAMES[k]: round(float(st[:, k].sum()) / tiles, 1) for k in range(1, 20)}}),
+                      "per_tile": {NAMES[k]: round(float(st[:, k].sum()) / tiles, 1) for k in range(1, 24)}}),
           flush=True)
