@@ -161,8 +161,9 @@ sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out,
  * them; the production library returns SAT_ERR_UNSUPPORTED. */
 sat_status_t sat_debug_stats(int64_t* out, int max_ctas, int* n_ctas, int* n_stats);
 
-/* Test/tuning hook: per-tile timeline of the most recent launch (libsat_stats.so only): out[2t] =
- * acquisition time, out[2t+1] = store-issue time of tile serial t, in %globaltimer nanoseconds. */
+/* Test/tuning hook: per-tile timeline of the most recent launch (libsat_stats.so only): out[8t + e]
+ * for tile serial t, %globaltimer ns: e = 0 acquired, 1 data landed (compute starts), 2 local
+ * aggregates published, 3 row walk resolved, 4 column walk resolved, 5 Step 4 done, 6 store issued. */
 sat_status_t sat_debug_trace(int64_t* out, int64_t max_tiles, int64_t* n_tiles);
 
 /* Free every cached workspace and staging buffer (synchronises the devices that own them). */

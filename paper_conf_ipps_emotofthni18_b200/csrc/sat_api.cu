@@ -418,7 +418,7 @@ sat_status_t compute_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ro
     p.trace = nullptr;
 #if SAT_STATS
     {
-        const size_t need = static_cast<size_t>(grid) * sat::kNumStats + 2 * static_cast<size_t>(pl.ntiles);
+        const size_t need = static_cast<size_t>(grid) * sat::kNumStats + 8 * static_cast<size_t>(pl.ntiles);
         if (w->stats_words < need) {
             if (w->stats) cudaFree(w->stats);
             SAT_CUDA(cudaMalloc(&w->stats, need * 8));
@@ -846,7 +846,7 @@ SAT_API sat_status_t sat_debug_trace(int64_t* out, int64_t max_tiles, int64_t* n
     const int64_t n = w->trace_tiles < max_tiles ? w->trace_tiles : max_tiles;
     SAT_CUDA(cudaStreamSynchronize(w->stream));
     SAT_CUDA(cudaMemcpy(out, w->stats + static_cast<size_t>(w->stats_ctas) * sat::kNumStats,
-                        static_cast<size_t>(n) * 16, cudaMemcpyDeviceToHost));
+                        static_cast<size_t>(n) * 64, cudaMemcpyDeviceToHost));
     *n_tiles = n;
     return SAT_OK;
 #else

@@ -321,6 +321,9 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
                 }
                 __syncwarp();
                 if (lane == 0) {
+#if SAT_STATS
+                    if (p.trace) p.trace[8LL * sm.info[x.s].t + (ROW ? 3 : 4)] = static_cast<long long>(globaltimer_ns());
+#endif
                     mbar_arrive(ROW ? &sm.rowwalk[x.s] : &sm.colwalk[x.s]);
                     WS_ST(ROW ? kWsRowTiles : kWsColTiles, 1);
 #if SAT_STATS
@@ -356,6 +359,9 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
     if (warp == 0 && lane == 0) { WS_ST(kWsFullWait, c1 - c0); WS_ST(kWsTiles, 1); }
     const TileInfo ti = sm.info[tq.s];
     if (ti.t >= p.ntiles) return false;
+#if SAT_STATS
+    if (p.trace && warp == 0 && lane == 0) p.trace[8LL * ti.t + 1] = static_cast<long long>(globaltimer_ns());
+#endif
     I = ti.I;
     J = ti.J;
     const long long tidx = static_cast<long long>(I) * p.C + J;
@@ -457,6 +463,9 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
     }
     SAT_CLK(c2);
     if (warp == 0 && lane == 0) WS_ST(kWsLocal, c2 - c1);
+#if SAT_STATS
+    if (p.trace && warp == NW - 1 && lane == 0) p.trace[8LL * ti.t + 2] = static_cast<long long>(globaltimer_ns());
+#endif
     return true;
 }
 
@@ -540,6 +549,9 @@ __device__ __forceinline__ void ws_finish(WsSmem<V, Cfg>& sm, const KParams<V>& 
             }
         }
     }
+#if SAT_STATS
+    if (p.trace && warp == 0 && lane == 0) p.trace[8LL * sm.info[tq.s].t + 5] = static_cast<long long>(globaltimer_ns());
+#endif
     __syncwarp();
     if (lane == 0) mbar_arrive(&sm.result[s]);
     SAT_CLK(c2);
@@ -619,7 +631,7 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 }
                 mbar_arrive(&sm.tfree[tq.s]);  // the tile slot (id, carries) is no longer needed
 #if SAT_STATS
-                if (p.trace) p.trace[2LL * ti.t + 1] = static_cast<long long>(globaltimer_ns());
+                if (p.trace) p.trace[8LL * ti.t + 6] = static_cast<long long>(globaltimer_ns());
 #endif
                 // release the stage as soon as its store has read the shared memory
                 if (stored) bulk_wait_read<0>();
@@ -666,7 +678,7 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 }
                 mbar_arrive(&sm.acq[ta.s]);
 #if SAT_STATS
-                if (p.trace && valid) p.trace[2LL * t] = static_cast<long long>(globaltimer_ns());
+                if (p.trace && valid) p.trace[8LL * t] = static_cast<long long>(globaltimer_ns());
 #endif
                 ta.next();
                 progress = true;
