@@ -344,7 +344,7 @@ def main():
                        "overhead_pct": (ms - memcpy_ms) / memcpy_ms * 100.0},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": load_ncu_traffic(workload), "peak_source": peak_src,
-                         "kernel": "sat_ws_kernel" if plan["family"] == 1 else "sat_tiles_kernel",
+                         "kernel": {2: "sat_tm_kernel", 1: "sat_ws_kernel"}.get(plan["family"], "sat_tiles_kernel"),
                          "bytes_per_elem": BYTES_PER_ELEM},
             "gpu_launches": args.steps * (1 if world == 1 else 4),
             "clocks": clk,

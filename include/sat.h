@@ -163,7 +163,8 @@ sat_status_t sat_debug_stats(int64_t* out, int max_ctas, int* n_ctas, int* n_sta
 
 /* Test/tuning hook: per-tile timeline of the most recent launch (libsat_stats.so only): out[8t + e]
  * for tile serial t, %globaltimer ns: e = 0 acquired, 1 data landed (compute starts), 2 local
- * aggregates published, 3 row walk resolved, 4 column walk resolved, 5 Step 4 done, 6 store issued. */
+ * aggregates published, 3 row walk resolved, 4 column walk resolved, 5 Step 4 done, 6 store issued,
+ * 7 TMA load issued (0 where a step does not apply to the variant). */
 sat_status_t sat_debug_trace(int64_t* out, int64_t max_tiles, int64_t* n_tiles);
 
 /* Free every cached workspace and staging buffer (synchronises the devices that own them). */

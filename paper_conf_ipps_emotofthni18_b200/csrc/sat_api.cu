@@ -18,6 +18,7 @@
 #include "sat_aux_kernels.cuh"
 #include "sat_kernel.cuh"
 #include "sat_ws_kernel.cuh"
+#include "sat_tm_kernel.cuh"
 
 #if defined(SAT_HAVE_NCCL_H)
 #include <nccl.h>
@@ -60,7 +61,7 @@ using PrepareFn = cudaError_t (*)(bool tma, bool carry, int* occupancy);
 
 struct Variant {
     int TR, TC, NW, STAGES;
-    int family;            // 1 = warp-specialised (sat_ws_kernel), 0 = classic (sat_tiles_kernel)
+    int family;            // 2 = TMEM-parked (sat_tm_kernel), 1 = warp-specialised (sat_ws_kernel), 0 = classic
     size_t smem;           // dynamic shared memory bytes (same for int32 / fp32)
     LaunchFn launch[2];    // [dtype]
     PrepareFn prepare[2];  // [dtype]
@@ -82,15 +83,26 @@ struct Family<sat::TileCfg<TR, TC, NW, ST>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_tiles_kernel<V, Cfg, TMA, CARRY>); }
 };
 
-template <int TR, int NW, int ST, int NT, int NQ>
-struct Family<sat::WsCfg<TR, NW, ST, NT, NQ>> {
-    using Cfg = sat::WsCfg<TR, NW, ST, NT, NQ>;
+template <int TR, int NW, int ST, int NT, int NQ, int FLAGS>
+struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
+    using Cfg = sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>;
     static constexpr int threads = Cfg::THREADS;
     static constexpr int family = 1;
     template <typename V>
     static constexpr size_t smem() { return sizeof(sat::WsSmem<V, Cfg>); }
     template <typename V, bool TMA, bool CARRY>
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
+};
+
+template <int NW, int IN, int NQ, int NT, int WPUB>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB>;
+    static constexpr int threads = Cfg::THREADS;
+    static constexpr int family = 2;
+    template <typename V>
+    static constexpr size_t smem() { return sizeof(sat::TmSmem<V, Cfg>); }
+    template <typename V, bool TMA, bool CARRY>
+    static void* kernel() { return reinterpret_cast<void*>(&sat::sat_tm_kernel<V, Cfg, TMA, CARRY>); }
 };
 
 template <typename V, typename F>
@@ -136,10 +148,10 @@ Variant make_variant() {
 
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
-        make_variant<sat::WsCfg<128, 16, 3, 1, 5>>(),  // 0: warp-specialised, 64 KiB tiles, 3 stages, 5-tile ring
-        make_variant<sat::WsCfg<128, 16, 3, 1, 3>>(),  // 1: ... tickets only as stages free up
-        make_variant<sat::WsCfg<128, 16, 3, 2, 6>>(),  // 2: ... 6-tile ring, two tiles per walker
-        make_variant<sat::WsCfg<64, 16, 6, 2, 8>>(),   // 3: warp-specialised, 32 KiB tiles, 6 stages, 8-tile ring
+        make_variant<sat::TmCfg<16, 2, 5>>(),  // 0: local SAT parked in TMEM, 2 input stages + output buffer, walkers publish
+        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 1: deferred finish, GSAT from registers
+        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch>>(),  // 2: 64 KiB tiles, 3 stages, TMA store
+        make_variant<sat::TmCfg<16, 2, 5, 1, 0>>(),  // 3: TMEM-parked, inclusive aggregates from the compute warps
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 4: classic, 32 KiB tiles, 2 stages
         make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 5: classic, 64 KiB tiles, 512 threads
     };

@@ -30,6 +30,47 @@ __device__ __forceinline__ V warp_inclusive_scan(V x, int lane) {
     return x;
 }
 
+// Exclusive prefix over the 32 lanes of a warp for N independent rows at once (tot[r] = this lane's
+// value in row r; ex[r] = sum over lanes < lane), through a transpose in shared memory instead of
+// N shuffle scans: G = 32/N lanes take one row each, sum N consecutive lane values serially, and
+// scan their G partial sums with log2(G) shuffles.  S: N*32 elements of warp-private, 16-byte
+// aligned scratch.  Same prefix sums as warp_inclusive_scan (different association for floats).
+template <typename V, int N>
+__device__ __forceinline__ void warp_rows_exclusive_smem(const V (&tot)[N], V (&ex)[N], V* S, int lane) {
+    static_assert(N >= 4 && N <= 32 && 32 % N == 0, "rows per transposed scan");
+    constexpr int G = 32 / N;
+#pragma unroll
+    for (int r = 0; r < N; ++r) S[r * 32 + lane] = tot[r];
+    __syncwarp();
+    const int row = lane / G, g = lane % G;
+    V x[N];
+#pragma unroll
+    for (int i = 0; i < N; i += 4) {
+        const uint4 q = *reinterpret_cast<const uint4*>(&S[row * 32 + g * N + i]);
+        x[i] = from_bits<V>(q.x); x[i + 1] = from_bits<V>(q.y); x[i + 2] = from_bits<V>(q.z); x[i + 3] = from_bits<V>(q.w);
+    }
+#pragma unroll
+    for (int i = 1; i < N; ++i) x[i] = x[i] + x[i - 1];
+    V inc = x[N - 1];
+#pragma unroll
+    for (int d = 1; d < G; d <<= 1) {
+        const V y = __shfl_up_sync(kFull, inc, d, G);
+        if (g >= d) inc = inc + y;
+    }
+    V base = __shfl_up_sync(kFull, inc, 1, G);
+    if (g == 0) base = V(0);
+    __syncwarp();
+#pragma unroll
+    for (int i = 0; i < N; i += 4) {
+        const V e0 = i == 0 ? base : base + x[i - 1];
+        *reinterpret_cast<uint4*>(&S[row * 32 + g * N + i]) =
+            make_uint4(to_bits(e0), to_bits(base + x[i]), to_bits(base + x[i + 1]), to_bits(base + x[i + 2]));
+    }
+    __syncwarp();
+#pragma unroll
+    for (int r = 0; r < N; ++r) ex[r] = S[r * 32 + lane];
+}
+
 template <typename V>
 __device__ __forceinline__ V warp_sum(V x) {
 #pragma unroll
@@ -85,6 +126,11 @@ __device__ __forceinline__ void tma_load_2d(void* smem_dst, const CUtensorMap* m
         : "memory");
 }
 
+// 2-D tile global -> L2 only (no shared memory, no completion): warms L2 ahead of the real load.
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int x, int y) {
+    asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global [%0, {%1, %2}];" ::"l"(map), "r"(x), "r"(y) : "memory");
+}
+
 // 2-D tile shared -> global; out-of-bounds box elements are not written (edge tiles, pitch pad).
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* smem_src, int x, int y) {
     asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(map), "r"(x),
@@ -99,6 +145,14 @@ __device__ __forceinline__ void tma_store_2d_hint(const CUtensorMap* map, const 
     asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%1, %2}], [%3], %4;" ::"l"(
                      map),
                  "r"(x), "r"(y), "r"(smem_addr(smem_src)), "l"(policy)
+                 : "memory");
+}
+
+// 16-byte global store with an L2 eviction policy (the streamed SAT output, written from registers).
+__device__ __forceinline__ void st_global_v4_hint(void* p, uint32_t a, uint32_t b, uint32_t c, uint32_t d,
+                                                  uint64_t pol) {
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.b32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "r"(a),
+                 "r"(b), "r"(c), "r"(d), "l"(pol)
                  : "memory");
 }
 
@@ -169,8 +223,9 @@ __device__ __forceinline__ void ld_relaxed2_p(const uint64_t* p, uint64_t& a, ui
 
 template <int E>
 __device__ __forceinline__ void st_words_p(uint64_t* p, const uint64_t (&w)[E], uint64_t pol) {
-    if constexpr (E == 1) {
-        st_relaxed_p(p, w[0], pol);
+    if constexpr (E % 2 != 0) {  // odd vectors are not 16-byte aligned per lane: scalar accesses
+#pragma unroll
+        for (int e = 0; e < E; ++e) st_relaxed_p(p + e, w[e], pol);
     } else {
 #pragma unroll
         for (int e = 0; e < E; e += 2) st_relaxed2_p(p + e, w[e], w[e + 1], pol);
@@ -179,8 +234,9 @@ __device__ __forceinline__ void st_words_p(uint64_t* p, const uint64_t (&w)[E], 
 
 template <int E>
 __device__ __forceinline__ void ld_words_p(const uint64_t* p, uint64_t (&w)[E], uint64_t pol) {
-    if constexpr (E == 1) {
-        w[0] = ld_relaxed_p(p, pol);
+    if constexpr (E % 2 != 0) {  // odd vectors are not 16-byte aligned per lane: scalar accesses
+#pragma unroll
+        for (int e = 0; e < E; ++e) w[e] = ld_relaxed_p(p + e, pol);
     } else {
 #pragma unroll
         for (int e = 0; e < E; e += 2) ld_relaxed2_p(p + e, w[e], w[e + 1], pol);
@@ -189,8 +245,9 @@ __device__ __forceinline__ void ld_words_p(const uint64_t* p, uint64_t (&w)[E], 
 
 template <int E>
 __device__ __forceinline__ void st_words(uint64_t* p, const uint64_t (&w)[E]) {
-    if constexpr (E == 1) {
-        st_relaxed(p, w[0]);
+    if constexpr (E % 2 != 0) {  // odd vectors are not 16-byte aligned per lane: scalar accesses
+#pragma unroll
+        for (int e = 0; e < E; ++e) st_relaxed(p + e, w[e]);
     } else {
 #pragma unroll
         for (int e = 0; e < E; e += 2) st_relaxed2(p + e, w[e], w[e + 1]);
@@ -199,8 +256,9 @@ __device__ __forceinline__ void st_words(uint64_t* p, const uint64_t (&w)[E]) {
 
 template <int E>
 __device__ __forceinline__ void ld_words(const uint64_t* p, uint64_t (&w)[E]) {
-    if constexpr (E == 1) {
-        w[0] = ld_relaxed(p);
+    if constexpr (E % 2 != 0) {  // odd vectors are not 16-byte aligned per lane: scalar accesses
+#pragma unroll
+        for (int e = 0; e < E; ++e) w[e] = ld_relaxed(p + e);
     } else {
 #pragma unroll
         for (int e = 0; e < E; e += 2) ld_relaxed2(p + e, w[e], w[e + 1]);

@@ -1,0 +1,532 @@
+// sat_tm_kernel.cuh -- single-pass SAT kernel for sm_100a with the local SAT parked in tensor memory.
+//
+// Same method, aggregates and walkers as sat_ws_kernel (1R1W-SKSS-LB of PAPER.md Sec. IV, P:182-249,
+// prefix-form slots, epoch-tagged status words; walkers: ws_walker).  What differs is where a tile
+// waits for its look-backs.  In sat_ws_kernel the compute warps hold a tile's local SAT in registers
+// and its input stage in shared memory until the walks land (~1 us per tile on B200 with HBM
+// saturated), which idles the warps and pins a 64 KiB stage.  Here:
+//
+//   * a tile's pixels are read out of their input stage into registers right away and the stage is
+//     handed back to the loader (the ring refills while the tile is still being computed);
+//   * after the local SAT and the local aggregates (Steps 2.A.1, 2.B.1) each compute warp
+//     parks its 8x128 block in TMEM (tcgen05.st; 2 slots x NW/4 warps x 32 columns, 256 of the
+//     512 columns) and goes on with the local SAT of the NEXT tile;
+//   * only then does it reload the parked block (tcgen05.ld), wait for the walks of the previous tile,
+//     publish its inclusive aggregates (Steps 2.A.3, 2.B.3, 3.1, 3.3) and apply Step 4 (rule
+//     P:150) into a dedicated output buffer, which the storer lane writes with a TMA 2-D store.
+//
+// Roles: loader lane (tickets + TMA loads), row / column walker warps (ws_walker), NW compute warps,
+// storer lane.  Barriers: acq / rowwalk / colwalk / tfree / result per tile slot (tile ring, NQ
+// deep); full / empty per input stage; ofree per output buffer.  The storer releases a tile slot
+// (tfree) once it has taken the tile's result, so every per-slot barrier is at most one phase ahead
+// of each of its waiters.
+#pragma once
+
+#include "sat_ws_kernel.cuh"
+
+namespace sat {
+
+template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1>
+struct TmCfg {
+    static constexpr int TR = 128, TC = 128, NW = NW_;
+    static constexpr int IN = IN_;    // input stages
+    static constexpr int STAGES = IN;
+    static constexpr int NQ = NQ_;    // tile ring
+    static constexpr int NT = NT_;    // tiles in flight per walker
+    static constexpr bool FAST = false;
+    static constexpr bool WPUB = WPUB_ != 0;  // the walkers publish the inclusive aggregates
+    static constexpr int RPW = TR / NW, ER = TR / 32, EC = TC / 32;
+    static constexpr int NREG = RPW * 4;         // 32-bit registers per thread parked per tile
+    static constexpr int TM_COLS_PER_SLOT = (NW / 4) * NREG;
+    static constexpr int TM_COLS = 2 * TM_COLS_PER_SLOT <= 32 ? 32 : 2 * TM_COLS_PER_SLOT <= 64 ? 64
+                                 : 2 * TM_COLS_PER_SLOT <= 128 ? 128 : 2 * TM_COLS_PER_SLOT <= 256 ? 256 : 512;
+    static constexpr int ROW_WARP = NW, COL_WARP = NW + 1, STORE_WARP = NW + 2, LOAD_WARP = NW + 3;
+    static constexpr int THREADS = (NW + 4) * 32;
+    static_assert(NW % 4 == 0 && TR % NW == 0 && RPW % 4 == 0, "compute warps cover the 4 TMEM lane quarters");
+    static_assert(NREG == 16 || NREG == 32, "tcgen05 32x32b.x16 / .x32 parking");
+    static_assert(2 * TM_COLS_PER_SLOT <= 512, "TMEM columns");
+    static_assert(IN >= 1 && NQ >= IN + 1 && NQ <= 16, "rings");
+};
+
+template <typename V, typename Cfg>
+struct TmSmem {
+    alignas(1024) V stage[Cfg::IN][Cfg::TR * Cfg::TC];  // input ring (TMA loads)
+    alignas(1024) V out[Cfg::TR * Cfg::TC];             // GSAT of one tile (TMA store source)
+    alignas(16) V band[2][Cfg::NW][Cfg::TC];
+    alignas(16) V rp[Cfg::NQ][Cfg::TR];
+    alignas(16) V cp[Cfg::NQ][Cfg::TC];
+    V corner[Cfg::NQ];
+    alignas(16) V lrs[Cfg::NQ][Cfg::TR];  // local row aggregates (prefix form) of the slot's tile (WPUB)
+    alignas(16) V lcs[Cfg::NQ][Cfg::TC];  // local column aggregates
+    alignas(8) uint64_t acq[Cfg::NQ];
+    uint64_t ldone[Cfg::NQ];  // lrs / lcs written (NW arrivals)
+    uint64_t rowwalk[Cfg::NQ];
+    uint64_t colwalk[Cfg::NQ];
+    uint64_t tfree[Cfg::NQ];
+    uint64_t result[Cfg::NQ];  // GSAT of the slot's tile is in `out` (NW arrivals)
+    uint64_t full[Cfg::IN];
+    uint64_t empty[Cfg::IN];   // input stage read into registers (NW arrivals)
+    uint64_t ofree;            // `out` read by the TMA store
+    alignas(16) TileInfo info[Cfg::NQ];
+    uint32_t epoch;
+    int end_n;
+    uint32_t tmem_base;
+};
+
+// ------------------------------------------------------------------ tcgen05 TMEM helpers
+__device__ __forceinline__ void tmem_alloc(uint32_t* dst_smem, int ncols) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_addr(dst_smem)),
+                 "r"(ncols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tmem_dealloc(uint32_t base, int ncols) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(base), "r"(ncols) : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// Park / reload the warp's RPW x 4 block: thread t of the warp uses TMEM lane (32 * (warp % 4) + t),
+// NREG consecutive columns from `col`.
+template <int N>
+__device__ __forceinline__ void tmem_st(uint32_t taddr, const uint32_t (&r)[N]);
+template <>
+__device__ __forceinline__ void tmem_st<32>(uint32_t taddr, const uint32_t (&r)[32]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31, %32};" ::"r"(taddr),
+        "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+        "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]), "r"(r[16]), "r"(r[17]), "r"(r[18]),
+        "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]),
+        "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
+        : "memory");
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+template <>
+__device__ __forceinline__ void tmem_st<16>(uint32_t taddr, const uint32_t (&r)[16]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15, %16};" ::"r"(taddr),
+        "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+        "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
+        : "memory");
+    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&r)[N]);
+template <>
+__device__ __forceinline__ void tmem_ld<32>(uint32_t taddr, uint32_t (&r)[32]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15, %16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+          "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),
+          "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+          "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr)
+        : "memory");
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+template <>
+__device__ __forceinline__ void tmem_ld<16>(uint32_t taddr, uint32_t (&r)[16]) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, "
+        "%15}, [%16];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+          "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+        : "r"(taddr)
+        : "memory");
+    asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+template <typename Cfg>
+__device__ __forceinline__ uint32_t tm_addr(uint32_t base, int warp, int slot) {
+    return base + (static_cast<uint32_t>(32 * (warp & 3)) << 16) +
+           static_cast<uint32_t>(slot * Cfg::TM_COLS_PER_SLOT + (warp >> 2) * Cfg::NREG);
+}
+
+// Step 1 + local SAT + Steps 2.A.1 / 2.B.1 of tile k (input stage sl, tile slot tq); parks the block in
+// TMEM slot k & 1.  Returns false at the end marker.
+template <typename V, typename Cfg, bool TMA>
+__device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p, const Slot<Cfg::IN>& sl,
+                                         const Slot<Cfg::NQ>& tq, uint32_t epoch, int warp, int lane) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
+    const int s = sl.s;
+    const int row0 = warp * RPW, col0 = lane * 4;
+    SAT_CLK(c0);
+    mbar_wait(&sm.full[s], sl.ph);
+    SAT_CLK(c1);
+    if (warp == 0 && lane == 0) { WS_ST(kWsFullWait, c1 - c0); WS_ST(kWsTiles, 1); }
+    const TileInfo ti = sm.info[tq.s];
+    if (ti.t >= p.ntiles) return false;
+#if SAT_STATS
+    if (p.trace && warp == 0 && lane == 0) p.trace[8LL * ti.t + 1] = static_cast<long long>(globaltimer_ns());
+#endif
+    const int I = ti.I, J = ti.J;
+    const long long tidx = static_cast<long long>(I) * p.C + J;
+    const int par = tq.k & 1;
+    V v[RPW][4];
+    if constexpr (TMA) {
+        const V* tile = sm.stage[s];
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const uint4 q = *reinterpret_cast<const uint4*>(&tile[(row0 + r) * TC + col0]);
+            v[r][0] = from_bits<V>(q.x); v[r][1] = from_bits<V>(q.y);
+            v[r][2] = from_bits<V>(q.z); v[r][3] = from_bits<V>(q.w);
+        }
+    } else {
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const long long gi = static_cast<long long>(I) * TR + row0 + r;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const long long gj = static_cast<long long>(J) * TC + col0 + c;
+                v[r][c] = (gi < p.rows && gj < p.cols) ? p.src[gi * p.pitch + gj] : V(0);
+            }
+        }
+    }
+    // the pixels are in registers: the loader may refill the stage now
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sm.empty[s]);
+    if (TMA && J == p.C - 1) {  // right edge: zero columns >= cols (16-byte TMA granules, reading R2)
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+            if (static_cast<long long>(J) * TC + col0 + c >= p.cols) {
+#pragma unroll
+                for (int r = 0; r < RPW; ++r) v[r][c] = V(0);
+            }
+    }
+    // local SAT: column prefix in the band, warp prefix-sum rows, bands above
+#pragma unroll
+    for (int r = 1; r < RPW; ++r)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + v[r - 1][c];
+#pragma unroll
+    for (int r = 0; r < RPW; ++r) {
+        v[r][1] = v[r][1] + v[r][0];
+        v[r][2] = v[r][2] + v[r][1];
+        v[r][3] = v[r][3] + v[r][2];
+        const V incl = warp_inclusive_scan(v[r][3], lane);
+        V excl = __shfl_up_sync(kFull, incl, 1);
+        if (lane == 0) excl = V(0);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + excl;
+    }
+    *reinterpret_cast<uint4*>(&sm.band[par][warp][col0]) =
+        make_uint4(to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
+    named_bar_sync(1, NW * 32);
+    {
+        const int tid = warp * 32 + lane;
+        if (tid < TC) {
+            V b[NW];
+#pragma unroll
+            for (int u = 0; u < NW; ++u) b[u] = sm.band[par][u][tid];
+            V run = V(0);
+#pragma unroll
+            for (int u = 0; u < NW; ++u) {
+                sm.band[par][u][tid] = run;
+                run = run + b[u];
+            }
+        }
+        named_bar_sync(1, NW * 32);
+        const uint4 q = *reinterpret_cast<const uint4*>(&sm.band[par][warp][col0]);
+        const V off[4] = {from_bits<V>(q.x), from_bits<V>(q.y), from_bits<V>(q.z), from_bits<V>(q.w)};
+#pragma unroll
+        for (int r = 0; r < RPW; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + off[c];
+    }
+    // Steps 2.A.1 / 2.B.1 (edge tiles publish inclusive at once: their carry is zero)
+    const uint64_t pol = policy_evict_last();
+    if (lane == 31) {
+        uint64_t* rs = p.row_slots + tidx * TR + row0;
+        const uint32_t kind = (J == 0) ? kIncl : kLocal;
+#pragma unroll
+        for (int r = 0; r < RPW; r += 2)
+            st_relaxed2_p(rs + r, pack(epoch, kind, to_bits(v[r][3])), pack(epoch, kind, to_bits(v[r + 1][3])), pol);
+    }
+    if (warp == NW - 1) {
+        uint64_t* cs = p.col_slots + tidx * TC + col0;
+        const uint32_t kind = (I == 0) ? kIncl : kLocal;
+        st_relaxed2_p(cs, pack(epoch, kind, to_bits(v[RPW - 1][0])), pack(epoch, kind, to_bits(v[RPW - 1][1])), pol);
+        st_relaxed2_p(cs + 2, pack(epoch, kind, to_bits(v[RPW - 1][2])), pack(epoch, kind, to_bits(v[RPW - 1][3])),
+                      pol);
+    }
+    if constexpr (Cfg::WPUB) {
+        if (lane == 31) {
+#pragma unroll
+            for (int r = 0; r < RPW; r += 4)
+                *reinterpret_cast<uint4*>(&sm.lrs[tq.s][row0 + r]) =
+                    make_uint4(to_bits(v[r][3]), to_bits(v[r + 1][3]), to_bits(v[r + 2][3]), to_bits(v[r + 3][3]));
+        }
+        if (warp == NW - 1)
+            *reinterpret_cast<uint4*>(&sm.lcs[tq.s][col0]) = make_uint4(
+                to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.ldone[tq.s]);
+    }
+    // park the block
+    uint32_t r32[Cfg::NREG];
+#pragma unroll
+    for (int r = 0; r < RPW; ++r)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) r32[r * 4 + c] = to_bits(v[r][c]);
+    tmem_st<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k & 1), r32);
+    SAT_CLK(c2);
+    if (warp == 0 && lane == 0) WS_ST(kWsLocal, c2 - c1);
+#if SAT_STATS
+    if (p.trace && warp == NW - 1 && lane == 0) p.trace[8LL * ti.t + 2] = static_cast<long long>(globaltimer_ns());
+#endif
+    return true;
+}
+
+// Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 and Step 4 of tile k (tile slot tq; its block parked in TMEM slot
+// k & 1), GSAT into the output buffer (use number `ou` of it).
+template <typename V, typename Cfg, bool TMA, bool CARRY>
+__device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& p, const Slot<Cfg::NQ>& tq,
+                                          uint32_t ou, uint32_t epoch, int warp, int lane) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
+    const int q = tq.s;
+    const int row0 = warp * RPW, col0 = lane * 4;
+    const TileInfo ti = sm.info[q];
+    const int I = ti.I, J = ti.J;
+    const long long tidx = static_cast<long long>(I) * p.C + J;
+    const uint64_t pol = policy_evict_last();
+    V v[RPW][4];
+    {
+        uint32_t r32[Cfg::NREG];
+        tmem_ld<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k & 1), r32);
+#pragma unroll
+        for (int r = 0; r < RPW; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) v[r][c] = from_bits<V>(r32[r * 4 + c]);
+    }
+    SAT_CLK(c0);
+    mbar_wait(&sm.rowwalk[q], tq.ph);
+    mbar_wait(&sm.colwalk[q], tq.ph);
+    SAT_CLK(c1);
+    if (warp == 0 && lane == 0) WS_ST(kWsWalkWait, c1 - c0);
+    V rt[RPW];
+#pragma unroll
+    for (int r = 0; r < RPW; r += 4) {
+        const uint4 u = *reinterpret_cast<const uint4*>(&sm.rp[q][row0 + r]);
+        rt[r] = from_bits<V>(u.x); rt[r + 1] = from_bits<V>(u.y); rt[r + 2] = from_bits<V>(u.z);
+        rt[r + 3] = from_bits<V>(u.w);
+    }
+    V cpv[4];
+    {
+        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[q][col0]);
+        cpv[0] = from_bits<V>(c4.x); cpv[1] = from_bits<V>(c4.y); cpv[2] = from_bits<V>(c4.z);
+        cpv[3] = from_bits<V>(c4.w);
+    }
+    const V corner = sm.corner[q];
+    if (!Cfg::WPUB && lane == 31 && J > 0) {
+        uint64_t* rs = p.row_slots + tidx * TR + row0;
+#pragma unroll
+        for (int r = 0; r < RPW; r += 2)
+            st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + rt[r])),
+                          pack(epoch, kIncl, to_bits(v[r + 1][3] + rt[r + 1])), pol);
+    }
+    if (!Cfg::WPUB && warp == NW - 1) {
+        if (I > 0) {
+            uint64_t* cs = p.col_slots + tidx * TC + col0;
+            st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + cpv[0])),
+                          pack(epoch, kIncl, to_bits(v[RPW - 1][1] + cpv[1])), pol);
+            st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + cpv[2])),
+                          pack(epoch, kIncl, to_bits(v[RPW - 1][3] + cpv[3])), pol);
+        }
+        if (lane == 31) {  // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
+            const V gls = v[RPW - 1][3] + rt[RPW - 1] + cpv[3];
+            st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(corner + gls)), pol);
+        }
+    }
+    V colterm[4];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) colterm[c] = cpv[c] + corner;
+    if constexpr (CARRY) {
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const long long gj = static_cast<long long>(J) * TC + col0 + c;
+            colterm[c] = colterm[c] + (gj < p.cols ? p.carry[gj] : V(0));
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < RPW; ++r)
+#pragma unroll
+        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + (rt[r] + colterm[c]);
+    const bool ragged = !TMA || ((J == p.C - 1) && (p.cols & 3) != 0);
+    if (!ragged) {
+        mbar_wait(&sm.ofree, (ou & 1u) ^ 1u);  // the previous tile's store has read `out`
+#pragma unroll
+        for (int r = 0; r < RPW; ++r)
+            *reinterpret_cast<uint4*>(&sm.out[(row0 + r) * TC + col0]) =
+                make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3]));
+        fence_proxy_async_smem();
+    } else {
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const long long gi = static_cast<long long>(I) * TR + row0 + r;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const long long gj = static_cast<long long>(J) * TC + col0 + c;
+                if (gi < p.rows && gj < p.cols) p.dst[gi * p.pitch + gj] = v[r][c];
+            }
+        }
+    }
+#if SAT_STATS
+    if (p.trace && warp == 0 && lane == 0) p.trace[8LL * ti.t + 5] = static_cast<long long>(globaltimer_ns());
+#endif
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sm.result[q]);
+    SAT_CLK(c2);
+    if (warp == 0 && lane == 0) WS_ST(kWsFinish, c2 - c1);
+}
+
+template <typename V, typename Cfg, bool TMA, bool CARRY>
+__global__ void __launch_bounds__(Cfg::THREADS, 1)
+sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant__ CUtensorMap map_out,
+              const KParams<V> p) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, IN = Cfg::IN;
+    constexpr uint32_t kTileBytes = TR * TC * sizeof(V);
+    extern __shared__ __align__(1024) unsigned char smem_raw[];
+    TmSmem<V, Cfg>& sm = *reinterpret_cast<TmSmem<V, Cfg>*>(smem_raw);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+#if SAT_STATS
+    if (threadIdx.x < kNumStats) ws_stats[threadIdx.x] = 0ull;
+#endif
+    if (warp == 0) tmem_alloc(&sm.tmem_base, Cfg::TM_COLS);
+    if (threadIdx.x == 32) {
+        sm.epoch = *reinterpret_cast<volatile unsigned int*>(&p.ctrl->epoch);
+        sm.end_n = 0x7fffffff;
+#pragma unroll
+        for (int q = 0; q < Cfg::NQ; ++q) {
+            mbar_init(&sm.acq[q], 1);
+            mbar_init(&sm.rowwalk[q], 1);
+            mbar_init(&sm.colwalk[q], 1);
+            mbar_init(&sm.tfree[q], 1);
+            mbar_init(&sm.result[q], NW);
+            mbar_init(&sm.ldone[q], NW);
+        }
+#pragma unroll
+        for (int s = 0; s < IN; ++s) {
+            mbar_init(&sm.full[s], 1);
+            mbar_init(&sm.empty[s], NW);
+        }
+        mbar_init(&sm.ofree, 1);
+        fence_mbar_init();
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t epoch = sm.epoch;
+
+    if (warp < NW) {
+        // ================================================================ compute warps
+        // local(0), then {local(k+1), finish(k)}: the walks of tile k run during local(k+1)
+        Slot<IN> sl;
+        Slot<Cfg::NQ> tq;
+        uint32_t ou = 0;  // uses of the output buffer so far
+        bool have = tm_local<V, Cfg, TMA>(sm, p, sl, tq, epoch, warp, lane);
+        while (have) {
+            Slot<IN> sl2 = sl;
+            Slot<Cfg::NQ> tq2 = tq;
+            sl2.next();
+            tq2.next();
+            const bool have2 = tm_local<V, Cfg, TMA>(sm, p, sl2, tq2, epoch, warp, lane);
+            const TileInfo ti = sm.info[tq.s];
+            const bool ragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
+            tm_finish<V, Cfg, TMA, CARRY>(sm, p, tq, ou, epoch, warp, lane);
+            if (!ragged) ++ou;
+            sl = sl2;
+            tq = tq2;
+            have = have2;
+        }
+        tc_fence_before();
+        named_bar_sync(2, NW * 32);
+        if (warp == 0) tmem_dealloc(sm.tmem_base, Cfg::TM_COLS);
+    } else if (warp == Cfg::ROW_WARP) {
+        ws_walker<V, Cfg, true>(sm, p, epoch, lane);
+    } else if (warp == Cfg::COL_WARP) {
+        ws_walker<V, Cfg, false>(sm, p, epoch, lane);
+    } else if (warp == Cfg::STORE_WARP) {
+        // ================================================================ storer (one lane)
+        if (lane == 0) {
+            if constexpr (TMA) prefetch_tensormap(&map_out);
+            const uint64_t spol = policy_evict_first();
+            for (Slot<Cfg::NQ> tq;; tq.next()) {
+                mbar_wait(&sm.acq[tq.s], tq.ph);
+                const TileInfo ti = sm.info[tq.s];
+                if (ti.t >= p.ntiles) break;
+                SAT_CLK(u0);
+                mbar_wait(&sm.result[tq.s], tq.ph);
+                // tile k is done with its slot (walks, carries, id): tile k + NQ may be acquired.  Released
+                // only here so that no barrier of the slot can run a phase ahead of this lane.
+                mbar_arrive(&sm.tfree[tq.s]);
+                SAT_CLK(u1);
+                WS_ST(kWsStResultWait, u1 - u0);
+                const bool ragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
+                if (!ragged) {
+                    tma_store_2d_hint(&map_out, sm.out, ti.J * TC, ti.I * TR, spol);
+                    bulk_commit();
+#if SAT_STATS
+                    if (p.trace) p.trace[8LL * ti.t + 6] = static_cast<long long>(globaltimer_ns());
+#endif
+                    bulk_wait_read<0>();
+                    mbar_arrive(&sm.ofree);
+                }
+                SAT_CLK(u2);
+                WS_ST(kWsStStore, u2 - u1);
+            }
+            if constexpr (TMA) bulk_wait_all();
+            ws_exit(p, epoch);
+        }
+    } else if (lane == 0) {
+        // ================================================================ loader (one lane)
+        const uint64_t policy = TMA ? policy_evict_first() : 0ull;
+        if constexpr (TMA) prefetch_tensormap(&map_in);
+        Slot<Cfg::NQ> ta, tl;
+        Slot<IN> sl;
+        bool acq_done = false;
+        while (true) {
+            bool progress = false;
+            if (!acq_done && (ta.k < Cfg::NQ || mbar_test(&sm.tfree[ta.s], ta.ph ^ 1u))) {
+                const int t = static_cast<int>(atomicAdd(&p.ctrl->counter, 1u));
+                const bool valid = t < p.ntiles;
+                TileInfo ti{t, 0, 0, 0};
+                if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
+                sm.info[ta.s] = ti;
+                if (!valid) {
+                    *reinterpret_cast<volatile int*>(&sm.end_n) = ta.k;
+                    acq_done = true;
+                }
+                mbar_arrive(&sm.acq[ta.s]);
+#if SAT_STATS
+                if (p.trace && valid) p.trace[8LL * t] = static_cast<long long>(globaltimer_ns());
+#endif
+                ta.next();
+                progress = true;
+            }
+            if (tl.k < ta.k && (sl.k < IN || mbar_test(&sm.empty[sl.s], sl.ph ^ 1u))) {
+                const TileInfo ti = sm.info[tl.s];
+                const bool valid = ti.t < p.ntiles;
+                if (TMA && valid) {
+                    mbar_arrive_expect_tx(&sm.full[sl.s], kTileBytes);
+                    tma_load_2d(sm.stage[sl.s], &map_in, &sm.full[sl.s], ti.J * TC, ti.I * TR, policy);
+#if SAT_STATS
+                    if (p.trace) p.trace[8LL * ti.t + 7] = static_cast<long long>(globaltimer_ns());
+#endif
+                } else {
+                    mbar_arrive(&sm.full[sl.s]);
+                }
+                tl.next();
+                sl.next();
+                progress = true;
+                if (!valid) break;
+            }
+            if (!progress) __nanosleep(32);
+        }
+    }
+}
+
+}  // namespace sat

@@ -35,7 +35,8 @@ namespace sat {
 enum WsStat {
     kWsTiles = 0, kWsFullWait, kWsLocal, kWsWalkWait, kWsFinish, kWsRowRounds, kWsColRounds,
     kWsStResultWait, kWsStStore, kWsLdIssue, kWsLdEmptyWait, kWsBandBar, kWsRowTiles, kWsColTiles,
-    kWsRowRoundCyc, kWsColRoundCyc, kWsRowResolve, kWsColResolve, kWsRowIdle, kWsColIdle, kWsRowLat, kWsColLat
+    kWsRowRoundCyc, kWsColRoundCyc, kWsRowResolve, kWsColResolve, kWsRowIdle, kWsColIdle, kWsRowLat, kWsColLat,
+    kWsFastHits, kWsScan
 };
 #if SAT_STATS
 __shared__ unsigned long long ws_stats[kNumStats];
@@ -84,11 +85,27 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-template <int TR_, int NW_, int STAGES_, int NT_, int NQ_>
+// Option bits of WsCfg (see the roles above).
+enum WsFlags : int {
+    kWsFast = 1,      // compute warps poll the direct predecessors themselves (walkers as fallback)
+    kWsDefer = 2,     // finish tile k after the local SAT of tile k+1 (local SAT parked in its stage)
+    kWsDirect = 4,    // GSAT stored from registers (no TMA store, no storer)
+    kWsPrefetch = 8,  // L2 prefetch of a tile's pixels as soon as it is acquired
+    kWsSmemScan = 16, // row scans transposed through shared memory instead of shuffle scans
+};
+
+template <int TR_, int NW_, int STAGES_, int NT_, int NQ_, int FLAGS_ = 0>
 struct WsCfg {
     static constexpr int TR = TR_, TC = 128, NW = NW_, STAGES = STAGES_;
     static constexpr int NQ = NQ_;        // tile ring: tiles acquired ahead of their data stage
     static constexpr int NT = NT_;        // tiles in flight per walker
+    static constexpr int FLAGS = FLAGS_;
+    static constexpr bool FAST = (FLAGS & kWsFast) != 0;
+    static constexpr bool DEFER = (FLAGS & kWsDefer) != 0;
+    static constexpr bool DIRECT = (FLAGS & kWsDirect) != 0;
+    static constexpr bool PREFETCH = (FLAGS & kWsPrefetch) != 0;
+    static constexpr bool SMEM_SCAN = (FLAGS & kWsSmemScan) != 0;
+    static constexpr bool WPUB = false;  // inclusive aggregates published by the compute warps
     static constexpr int RPW = TR / NW;   // rows per compute-warp band
     static constexpr int ER = TR / 32;    // row-vector elements per walker lane
     static constexpr int EC = TC / 32;    // column-vector elements per walker lane
@@ -97,8 +114,10 @@ struct WsCfg {
     static constexpr int MINB = 1;
     static_assert(TR % NW == 0 && TR % 32 == 0, "tile shape");
     static_assert(RPW % 2 == 0, "row slots are published in pairs");
-    static_assert(ER == 1 || ER % 2 == 0, "row vector split");
     static_assert(STAGES >= 2 && STAGES <= 8 && NT >= 1 && NQ >= STAGES && NQ <= 16, "rings");
+    static_assert(!FAST || (NW >= 3 && ER <= 4 && ER % 2 == 0), "fast-path poll warps 0, 1, NW-1");
+    static_assert(!(FAST && DEFER), "the fast-path poll registers would not survive the deferred finish");
+    static_assert(!(FAST && DIRECT), "fast path releases tile slots through the storer");
 };
 
 // Two rings: the data stages (tile k's pixels live in stage k % STAGES) and the tile ring (tile k's
@@ -111,6 +130,11 @@ struct WsSmem {
     alignas(16) V rp[Cfg::NQ][Cfg::TR];  // row carry    prefix_i GRS(I,J-1)
     alignas(16) V cp[Cfg::NQ][Cfg::TC];  // column carry prefix_j GCS(I-1,J)
     V corner[Cfg::NQ];                   // GS(I-1,J-1)
+    alignas(16) V rpf[Cfg::TR];          // fast path: the same carries read from inclusive predecessors
+    alignas(16) V cpf[Cfg::TC];
+    V cornerf;
+    int fok[3];                          // fast path: row / column / corner predecessor inclusive
+    int fdone[Cfg::NQ];                  // tile slot resolved by the fast path (walkers may stop)
     alignas(8) uint64_t acq[Cfg::NQ];    // tile id written (tile ring)
     uint64_t rowwalk[Cfg::NQ];
     uint64_t colwalk[Cfg::NQ];
@@ -137,8 +161,8 @@ struct Slot {
 
 // Walkers only wait for their next tile's acquisition; once the loader has drawn the end marker they
 // stop.  Returns false when tile k will never exist.
-template <typename V, typename Cfg>
-__device__ __forceinline__ bool wait_acquired(WsSmem<V, Cfg>& sm, int s, uint32_t parity, int k) {
+template <typename SM>
+__device__ __forceinline__ bool wait_acquired(SM& sm, int s, uint32_t parity, int k) {
     while (!mbar_try(&sm.acq[s], parity))
         if (k >= *reinterpret_cast<volatile int*>(&sm.end_n)) return false;
     return true;
@@ -173,13 +197,16 @@ __device__ __forceinline__ bool lb_consume(uint32_t& pending, int& pos, V (&acc)
     return progress;
 }
 
-template <typename V, typename Cfg, bool ROW>
-__device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
+// (SM: WsSmem, or any shared-memory layout with the same walker-facing members: acq, info, end_n,
+// rp, cp, corner, rowwalk, colwalk.)
+template <typename V, typename Cfg, bool ROW, typename SM>
+__device__ __forceinline__ void ws_walker(SM& sm, const KParams<V>& p, uint32_t epoch, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC;
     constexpr int E = ROW ? Cfg::ER : Cfg::EC;
     constexpr int NT = Cfg::NT;
     struct Walk {
         int active, s, I, J, pos;
+        uint32_t ph;
         uint32_t pend;
         V acc[E];
         V dacc;
@@ -219,6 +246,7 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
             Walk& x = wk[w];
             x.active = 1;
             x.s = next.s;
+            x.ph = next.ph;
             x.I = ti.I;
             x.J = ti.J;
             x.pos = ROW ? ti.J - 1 : ti.I - 1;
@@ -242,11 +270,18 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
         }
         // ---- one polling round: issue every load first ...
         uint64_t w0[NT][E], w1[NT][E], wd[NT];
+        bool fd[NT];
 #pragma unroll
         for (int w = 0; w < NT; ++w) {
             const Walk& x = wk[w];
             wd[w] = 0;
+            fd[w] = false;
             if (!x.active) continue;
+            if constexpr (Cfg::FAST) {
+                // the compute warps found the direct predecessors inclusive: nothing left to walk
+                fd[w] = __shfl_sync(kFull, *reinterpret_cast<volatile int*>(&sm.fdone[x.s]), 0) != 0;
+                if (fd[w]) continue;
+            }
             if (x.pend) {
                 if (ROW) {
                     const long long base = static_cast<long long>(x.I) * p.C;
@@ -290,6 +325,12 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
         for (int w = 0; w < NT; ++w) {
             Walk& x = wk[w];
             if (!x.active) continue;
+            if (fd[w]) {
+                if (lane == 0) mbar_arrive(ROW ? &sm.rowwalk[x.s] : &sm.colwalk[x.s]);
+                x.active = 0;
+                progress = true;
+                continue;
+            }
             if (x.pend) progress |= lb_consume<V, E>(x.pend, x.pos, x.acc, w0[w], w1[w], x.pos >= 1, epoch);
             if (ROW && !x.ddone) {
                 // Step 3.2: GS(I-1,J-1) = GS(I-k,J-k) + sum of GLS of the tiles between
@@ -311,6 +352,29 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
                 }
             }
             if (x.ddone && __all_sync(kFull, x.pend == 0u)) {
+                if constexpr (Cfg::WPUB) {
+                    // Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 from here, as soon as both the walk and the tile's
+                    // local aggregates (lrs / lcs, kept in smem by the compute warps) are in: successors
+                    // need not wait for the compute warps to reach the tile's Step 4.
+                    mbar_wait(&sm.ldone[x.s], x.ph);
+                    const long long tidx = static_cast<long long>(x.I) * p.C + x.J;
+                    V l[E];
+#pragma unroll
+                    for (int e = 0; e < E; ++e) l[e] = ROW ? sm.lrs[x.s][lane * E + e] : sm.lcs[x.s][lane * E + e];
+                    uint64_t wv[E];
+#pragma unroll
+                    for (int e = 0; e < E; ++e) wv[e] = pack(epoch, kIncl, to_bits(l[e] + x.acc[e]));
+                    if (ROW) {
+                        if (x.J > 0) st_words_p<E>(p.row_slots + tidx * TR + lane * E, wv, pol);
+                        mbar_wait(&sm.colwalk[x.s], x.ph);  // the column carry of the same tile
+                        if (lane == 31) {  // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
+                            const V gls = l[E - 1] + x.acc[E - 1] + sm.cp[x.s][TC - 1];
+                            st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(x.dacc + gls)), pol);
+                        }
+                    } else if (x.I > 0) {
+                        st_words_p<E>(p.col_slots + tidx * TC + lane * E, wv, pol);
+                    }
+                }
                 if (ROW) {
 #pragma unroll
                     for (int e = 0; e < E; ++e) sm.rp[x.s][lane * E + e] = x.acc[e];
@@ -348,8 +412,8 @@ __device__ __forceinline__ void ws_walker(WsSmem<V, Cfg>& sm, const KParams<V>& 
 // at the end marker.
 template <typename V, typename Cfg, bool TMA>
 __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p, V (&v)[Cfg::RPW][4],
-                                         const Slot<Cfg::STAGES>& sl, const Slot<Cfg::NQ>& tq, int& I, int& J,
-                                         uint32_t epoch, int warp, int lane) {
+                                         uint64_t (&fw)[4], const Slot<Cfg::STAGES>& sl, const Slot<Cfg::NQ>& tq,
+                                         int& I, int& J, uint32_t epoch, int warp, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
     const int s = sl.s;
     const int row0 = warp * RPW, col0 = lane * 4;
@@ -366,6 +430,28 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
     J = ti.J;
     const long long tidx = static_cast<long long>(I) * p.C + J;
     const int par = sl.k & 1;
+    const uint64_t pol = policy_evict_last();
+    if constexpr (Cfg::FAST) {
+        // Fast path of Steps 2.A.2 / 2.B.2 / 3.2: the direct predecessors (I,J-1), (I-1,J), (I-1,J-1)
+        // have usually published their inclusive aggregates by now; poll them once, here, so the
+        // round trip overlaps the local SAT (consumed in ws_finish; the walkers are the fallback).
+        constexpr int ER = Cfg::ER;
+        if (warp == 0) {
+            if (J > 0) {
+#pragma unroll
+                for (int e = 0; e < ER; e += 2)
+                    ld_relaxed2_p(p.row_slots + (tidx - 1) * TR + lane * ER + e, fw[e], fw[e + 1], pol);
+            }
+        } else if (warp == NW - 1) {
+            if (I > 0) {
+                const uint64_t* cs = p.col_slots + (tidx - p.C) * TC + col0;
+                ld_relaxed2_p(cs, fw[0], fw[1], pol);
+                ld_relaxed2_p(cs + 2, fw[2], fw[3], pol);
+            }
+        } else if (warp == 1 && lane == 0 && I > 0 && J > 0) {
+            fw[0] = ld_relaxed_p(p.corner_slots + tidx - p.C - 1, pol);
+        }
+    }
 
     // ---- Step 1 (data in smem, or read from global on the generic path): tile -> registers
     if constexpr (TMA) {
@@ -396,29 +482,56 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
         }
     }
 
+    if constexpr (Cfg::DIRECT && !Cfg::DEFER && !Cfg::SMEM_SCAN) {
+        // the tile now lives in registers: hand the stage back to the loader at once
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.empty[s]);
+    }
+
     // ---- local SAT: column prefix inside the warp's band, row scans with the warp prefix-sum
     //      algorithm, then the SAT rows of the bands above
 #pragma unroll
     for (int r = 1; r < RPW; ++r)
 #pragma unroll
         for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + v[r - 1][c];
+    if constexpr (Cfg::SMEM_SCAN) {
+        // scratch: this warp's own rows of the stage (already in registers, rewritten only in ws_finish)
+        V tot[RPW], ex[RPW];
 #pragma unroll
-    for (int r = 0; r < RPW; ++r) {
-        v[r][1] = v[r][1] + v[r][0];
-        v[r][2] = v[r][2] + v[r][1];
-        v[r][3] = v[r][3] + v[r][2];
-        const V incl = warp_inclusive_scan(v[r][3], lane);
-        V excl = __shfl_up_sync(kFull, incl, 1);
-        if (lane == 0) excl = V(0);
+        for (int r = 0; r < RPW; ++r) {
+            v[r][1] = v[r][1] + v[r][0];
+            v[r][2] = v[r][2] + v[r][1];
+            v[r][3] = v[r][3] + v[r][2];
+            tot[r] = v[r][3];
+        }
+        warp_rows_exclusive_smem<V, RPW>(tot, ex, sm.stage[s] + row0 * TC, lane);
 #pragma unroll
-        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + excl;
+        for (int r = 0; r < RPW; ++r)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + ex[r];
+        if constexpr (Cfg::DIRECT && !Cfg::DEFER) {
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&sm.empty[s]);
+        }
+    } else {
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            v[r][1] = v[r][1] + v[r][0];
+            v[r][2] = v[r][2] + v[r][1];
+            v[r][3] = v[r][3] + v[r][2];
+            const V incl = warp_inclusive_scan(v[r][3], lane);
+            V excl = __shfl_up_sync(kFull, incl, 1);
+            if (lane == 0) excl = V(0);
+#pragma unroll
+            for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + excl;
+        }
     }
     *reinterpret_cast<uint4*>(&sm.band[par][warp][col0]) =
         make_uint4(to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
     SAT_CLK(cb0);
     named_bar_sync(1, NW * 32);
     SAT_CLK(cb1);
-    if (warp == 0 && lane == 0) WS_ST(kWsBandBar, cb1 - cb0);
+    if (warp == 0 && lane == 0) { WS_ST(kWsBandBar, cb1 - cb0); WS_ST(kWsScan, cb0 - c1); }
     {
         // column-wise exclusive scan of the NW band bottoms, in place, by the first TC compute
         // threads (one column each); then every warp reads its band's offset in one 16-byte load
@@ -446,7 +559,6 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
     // ---- Steps 2.A.1 / 2.B.1: local aggregates (prefix form) from the owning lanes: the last column
     //      (lane 31 of every warp) and the bottom row (last warp).  Edge tiles publish inclusive at
     //      once: their carry is zero.
-    const uint64_t pol = policy_evict_last();
     if (lane == 31) {
         uint64_t* rs = p.row_slots + tidx * TR + row0;
         const uint32_t kind = (J == 0) ? kIncl : kLocal;
@@ -461,6 +573,14 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
         st_relaxed2_p(cs + 2, pack(epoch, kind, to_bits(v[RPW - 1][2])), pack(epoch, kind, to_bits(v[RPW - 1][3])),
                       pol);
     }
+    if constexpr (Cfg::DEFER) {
+        // park the local SAT in the tile's stage; ws_finish reloads it after the next tile's local
+        V* tile = sm.stage[s];
+#pragma unroll
+        for (int r = 0; r < RPW; ++r)
+            *reinterpret_cast<uint4*>(&tile[(row0 + r) * TC + col0]) =
+                make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3]));
+    }
     SAT_CLK(c2);
     if (warp == 0 && lane == 0) WS_ST(kWsLocal, c2 - c1);
 #if SAT_STATS
@@ -472,49 +592,125 @@ __device__ __forceinline__ bool ws_local(WsSmem<V, Cfg>& sm, const KParams<V>& p
 // Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 and Step 4 for the tile in stage sl.s whose local SAT is in `v`.
 template <typename V, typename Cfg, bool TMA, bool CARRY>
 __device__ __forceinline__ void ws_finish(WsSmem<V, Cfg>& sm, const KParams<V>& p, V (&v)[Cfg::RPW][4],
-                                          const Slot<Cfg::STAGES>& sl, const Slot<Cfg::NQ>& tq, int I, int J,
-                                          uint32_t epoch, int warp, int lane) {
+                                          const uint64_t (&fw)[4], const Slot<Cfg::STAGES>& sl,
+                                          const Slot<Cfg::NQ>& tq, int I, int J, uint32_t epoch, int warp,
+                                          int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
     const int s = sl.s, q = tq.s;
     const int row0 = warp * RPW, col0 = lane * 4;
     const long long tidx = static_cast<long long>(I) * p.C + J;
     const uint64_t pol = policy_evict_last();
+#if SAT_STATS
+    const int trace_t = sm.info[q].t;  // the slot may be reacquired once released below
+#endif
     SAT_CLK(c0);
-    mbar_wait(&sm.rowwalk[q], tq.ph);
-    mbar_wait(&sm.colwalk[q], tq.ph);
+    bool fast = false;
+    if constexpr (Cfg::FAST) {
+        // An inclusive predecessor word IS the carry (prefix-form slots): if all three are inclusive
+        // the walks are not needed.  Decided CTA-wide (all or nothing) after one barrier.
+        constexpr int ER = Cfg::ER;
+        auto incl_ok = [&](uint64_t w) { return word_ready(w, epoch) && word_kind(w) == kIncl; };
+        if (warp == 0) {
+            bool ok = true;
+            V val[ER];
+#pragma unroll
+            for (int e = 0; e < ER; ++e) {
+                val[e] = (J > 0) ? from_bits<V>(static_cast<uint32_t>(fw[e])) : V(0);
+                if (J > 0) ok = ok && incl_ok(fw[e]);
+            }
+            ok = __all_sync(kFull, ok);
+            if (ok) {
+#pragma unroll
+                for (int e = 0; e < ER; ++e) sm.rpf[lane * ER + e] = val[e];
+            }
+            if (lane == 0) sm.fok[0] = ok;
+        } else if (warp == NW - 1) {
+            bool ok = true;
+            V val[4];
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                val[c] = (I > 0) ? from_bits<V>(static_cast<uint32_t>(fw[c])) : V(0);
+                if (I > 0) ok = ok && incl_ok(fw[c]);
+            }
+            ok = __all_sync(kFull, ok);
+            if (ok)
+                *reinterpret_cast<uint4*>(&sm.cpf[col0]) =
+                    make_uint4(to_bits(val[0]), to_bits(val[1]), to_bits(val[2]), to_bits(val[3]));
+            if (lane == 0) sm.fok[1] = ok;
+        } else if (warp == 1 && lane == 0) {
+            const bool edge = (I == 0 || J == 0);
+            const bool ok = edge || incl_ok(fw[0]);
+            sm.cornerf = edge ? V(0) : from_bits<V>(static_cast<uint32_t>(fw[0]));
+            sm.fok[2] = ok;
+        }
+        named_bar_sync(2, NW * 32);
+        fast = sm.fok[0] && sm.fok[1] && sm.fok[2];
+        if (warp == 0 && lane == 0) {
+            if (fast) *reinterpret_cast<volatile int*>(&sm.fdone[q]) = 1;
+            WS_ST(kWsFastHits, fast ? 1 : 0);
+        }
+    }
+    if (!fast) {
+        mbar_wait(&sm.rowwalk[q], tq.ph);
+        mbar_wait(&sm.colwalk[q], tq.ph);
+    }
     SAT_CLK(c1);
     if (warp == 0 && lane == 0) WS_ST(kWsWalkWait, c1 - c0);
+    const V* rps = fast ? sm.rpf : sm.rp[q];
+    const V* cps = fast ? sm.cpf : sm.cp[q];
     V rt[RPW];
 #pragma unroll
-    for (int r = 0; r < RPW; ++r) rt[r] = sm.rp[q][row0 + r];
+    for (int r = 0; r < RPW; ++r) rt[r] = rps[row0 + r];
     V cpv[4];
     {
-        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[q][col0]);
+        const uint4 c4 = *reinterpret_cast<const uint4*>(&cps[col0]);
         cpv[0] = from_bits<V>(c4.x); cpv[1] = from_bits<V>(c4.y); cpv[2] = from_bits<V>(c4.z);
         cpv[3] = from_bits<V>(c4.w);
     }
-    const V corner = sm.corner[q];
-    // inclusive aggregates, from the lanes that hold the local ones
-    if (lane == 31 && J > 0) {
-        uint64_t* rs = p.row_slots + tidx * TR + row0;
+    const V corner = fast ? sm.cornerf : sm.corner[q];
+    if constexpr (Cfg::DEFER) {
+        const V* tile = sm.stage[s];
 #pragma unroll
-        for (int r = 0; r < RPW; r += 2)
-            st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + rt[r])),
-                          pack(epoch, kIncl, to_bits(v[r + 1][3] + rt[r + 1])), pol);
-    }
-    if (warp == NW - 1) {
-        if (I > 0) {
-            uint64_t* cs = p.col_slots + tidx * TC + col0;
-            st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + cpv[0])),
-                          pack(epoch, kIncl, to_bits(v[RPW - 1][1] + cpv[1])), pol);
-            st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + cpv[2])),
-                          pack(epoch, kIncl, to_bits(v[RPW - 1][3] + cpv[3])), pol);
-        }
-        if (lane == 31) {  // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
-            const V gls = v[RPW - 1][3] + rt[RPW - 1] + cpv[3];
-            st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(corner + gls)), pol);
+        for (int r = 0; r < RPW; ++r) {
+            const uint4 u = *reinterpret_cast<const uint4*>(&tile[(row0 + r) * TC + col0]);
+            v[r][0] = from_bits<V>(u.x); v[r][1] = from_bits<V>(u.y);
+            v[r][2] = from_bits<V>(u.z); v[r][3] = from_bits<V>(u.w);
         }
     }
+    if constexpr (Cfg::DIRECT) {
+        // carries are in registers, and (deferred) so is the local SAT: release the tile slot and stage
+        __syncwarp();
+        if (lane == 0) {
+            mbar_arrive(&sm.tfree[q]);
+            if constexpr (Cfg::DEFER) mbar_arrive(&sm.empty[s]);
+        }
+    }
+    // inclusive aggregates (Steps 2.A.3, 2.B.3, 3.1, 3.3), from the lanes that hold the local ones, at
+    // once (successors are waiting for them; publishing after the stage hand-off measured no faster)
+    V rinc[RPW], cinc[4];
+#pragma unroll
+    for (int r = 0; r < RPW; ++r) rinc[r] = v[r][3] + rt[r];
+#pragma unroll
+    for (int c = 0; c < 4; ++c) cinc[c] = v[RPW - 1][c] + cpv[c];
+    const V gs = corner + (v[RPW - 1][3] + rt[RPW - 1] + cpv[3]);  // GS = GS(I-1,J-1) + GLS
+    auto publish_incl = [&]() {
+        if (lane == 31 && J > 0) {
+            uint64_t* rs = p.row_slots + tidx * TR + row0;
+#pragma unroll
+            for (int r = 0; r < RPW; r += 2)
+                st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(rinc[r])), pack(epoch, kIncl, to_bits(rinc[r + 1])),
+                              pol);
+        }
+        if (warp == NW - 1) {
+            if (I > 0) {
+                uint64_t* cs = p.col_slots + tidx * TC + col0;
+                st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(cinc[0])), pack(epoch, kIncl, to_bits(cinc[1])), pol);
+                st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(cinc[2])), pack(epoch, kIncl, to_bits(cinc[3])), pol);
+            }
+            if (lane == 31) st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(gs)), pol);
+        }
+    };
+    publish_incl();
     // GSAT(I,J) = localSAT + rp[i] + cp[j] + corner (+ carry[j])
     V colterm[4];
 #pragma unroll
@@ -531,7 +727,24 @@ __device__ __forceinline__ void ws_finish(WsSmem<V, Cfg>& sm, const KParams<V>& 
 #pragma unroll
         for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + (rt[r] + colterm[c]);
     const bool ragged = !TMA || ((J == p.C - 1) && (p.cols & 3) != 0);
-    if (!ragged) {
+    if constexpr (Cfg::DIRECT && TMA) {
+        // 16-byte aligned rows (TMA path preconditions): one vector store per row chunk
+        const uint64_t spol = policy_evict_first();
+        const long long gj0 = static_cast<long long>(J) * TC + col0;
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const long long gi = static_cast<long long>(I) * TR + row0 + r;
+            if (gi >= p.rows) continue;
+            V* dst = p.dst + gi * p.pitch + gj0;
+            if (gj0 + 3 < p.cols) {
+                st_global_v4_hint(dst, to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3]), spol);
+            } else {
+#pragma unroll
+                for (int c = 0; c < 4; ++c)
+                    if (gj0 + c < p.cols) dst[c] = v[r][c];
+            }
+        }
+    } else if (!ragged) {
         V* tile = sm.stage[s];
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
@@ -550,12 +763,33 @@ __device__ __forceinline__ void ws_finish(WsSmem<V, Cfg>& sm, const KParams<V>& 
         }
     }
 #if SAT_STATS
-    if (p.trace && warp == 0 && lane == 0) p.trace[8LL * sm.info[tq.s].t + 5] = static_cast<long long>(globaltimer_ns());
+    if (p.trace && warp == 0 && lane == 0) p.trace[8LL * trace_t + 5] = static_cast<long long>(globaltimer_ns());
 #endif
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&sm.result[s]);
+    if constexpr (!Cfg::DIRECT) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.result[s]);
+    }
     SAT_CLK(c2);
     if (warp == 0 && lane == 0) WS_ST(kWsFinish, c2 - c1);
+}
+
+// Kernel exit (one thread per CTA, after all its tiles are stored): the last CTA out resets the ticket
+// counter and advances the epoch for the next launch (R9).
+template <typename V>
+__device__ __forceinline__ void ws_exit(const KParams<V>& p, uint32_t epoch) {
+    __threadfence();
+    const unsigned int done = atomicAdd(&p.ctrl->exit_count, 1u);
+#if SAT_STATS
+    if (p.stats)
+        for (int k = 0; k < kNumStats; ++k)
+            p.stats[static_cast<long long>(blockIdx.x) * kNumStats + k] = static_cast<long long>(ws_stats[k]);
+#endif
+    if (done == gridDim.x - 1) {
+        p.ctrl->counter = 0u;
+        p.ctrl->exit_count = 0u;
+        p.ctrl->epoch = (epoch >= kEpochMax) ? 1u : epoch + 1u;
+        __threadfence();
+    }
 }
 
 template <typename V, typename Cfg, bool TMA, bool CARRY>
@@ -579,13 +813,13 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
             mbar_init(&sm.acq[q], 1);
             mbar_init(&sm.rowwalk[q], 1);
             mbar_init(&sm.colwalk[q], 1);
-            mbar_init(&sm.tfree[q], 1);
+            mbar_init(&sm.tfree[q], Cfg::DIRECT ? NW : 1);
         }
 #pragma unroll
         for (int s = 0; s < STAGES; ++s) {
             mbar_init(&sm.full[s], 1);
             mbar_init(&sm.result[s], NW);
-            mbar_init(&sm.empty[s], 1);
+            mbar_init(&sm.empty[s], Cfg::DIRECT ? NW : 1);
         }
         fence_mbar_init();
     }
@@ -595,16 +829,46 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
     if (warp < NW) {
         // ================================================================ compute warps
         V v[RPW][4];
+        uint64_t fw[4] = {0ull, 0ull, 0ull, 0ull};
         Slot<STAGES> sl;
-        for (Slot<Cfg::NQ> tq;; tq.next(), sl.next()) {
+        Slot<Cfg::NQ> tq;
+        if constexpr (Cfg::DEFER) {
+            // local(k+1) runs while the walks of tile k finish: local(0), {local(k+1), finish(k)}...
             int I, J;
-            if (!ws_local<V, Cfg, TMA>(sm, p, v, sl, tq, I, J, epoch, warp, lane)) break;
-            ws_finish<V, Cfg, TMA, CARRY>(sm, p, v, sl, tq, I, J, epoch, warp, lane);
+            bool have = ws_local<V, Cfg, TMA>(sm, p, v, fw, sl, tq, I, J, epoch, warp, lane);
+            while (have) {
+                Slot<STAGES> sl2 = sl;
+                Slot<Cfg::NQ> tq2 = tq;
+                sl2.next();
+                tq2.next();
+                int I2, J2;
+                const bool have2 = ws_local<V, Cfg, TMA>(sm, p, v, fw, sl2, tq2, I2, J2, epoch, warp, lane);
+                ws_finish<V, Cfg, TMA, CARRY>(sm, p, v, fw, sl, tq, I, J, epoch, warp, lane);
+                sl = sl2;
+                tq = tq2;
+                I = I2;
+                J = J2;
+                have = have2;
+            }
+        } else {
+            for (;; tq.next(), sl.next()) {
+                int I, J;
+                if (!ws_local<V, Cfg, TMA>(sm, p, v, fw, sl, tq, I, J, epoch, warp, lane)) break;
+                ws_finish<V, Cfg, TMA, CARRY>(sm, p, v, fw, sl, tq, I, J, epoch, warp, lane);
+            }
+        }
+        if constexpr (Cfg::DIRECT) {
+            __threadfence();
+            named_bar_sync(3, (NW + 1) * 32);
         }
     } else if (warp == Cfg::ROW_WARP) {
         ws_walker<V, Cfg, true>(sm, p, epoch, lane);
     } else if (warp == Cfg::COL_WARP) {
         ws_walker<V, Cfg, false>(sm, p, epoch, lane);
+    } else if (warp == Cfg::STORE_WARP && Cfg::DIRECT) {
+        // compute warps store from registers: this warp only runs the exit protocol once they are done
+        named_bar_sync(3, (NW + 1) * 32);
+        if (lane == 0) ws_exit(p, epoch);
     } else if (warp == Cfg::STORE_WARP) {
         // ================================================================ storer (one lane)
         if (lane == 0) {
@@ -629,6 +893,9 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                         stored = true;
                     }
                 }
+                // the walkers may still be winding down a tile the fast path resolved
+                mbar_wait(&sm.rowwalk[tq.s], tq.ph);
+                mbar_wait(&sm.colwalk[tq.s], tq.ph);
                 mbar_arrive(&sm.tfree[tq.s]);  // the tile slot (id, carries) is no longer needed
 #if SAT_STATS
                 if (p.trace) p.trace[8LL * ti.t + 6] = static_cast<long long>(globaltimer_ns());
@@ -640,19 +907,7 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 WS_ST(kWsStStore, u2 - u1);
             }
             if constexpr (TMA) bulk_wait_all();
-            __threadfence();
-            const unsigned int done = atomicAdd(&p.ctrl->exit_count, 1u);
-#if SAT_STATS
-            if (p.stats)
-                for (int k = 0; k < kNumStats; ++k)
-                    p.stats[static_cast<long long>(blockIdx.x) * kNumStats + k] = static_cast<long long>(ws_stats[k]);
-#endif
-            if (done == gridDim.x - 1) {
-                p.ctrl->counter = 0u;
-                p.ctrl->exit_count = 0u;
-                p.ctrl->epoch = (epoch >= kEpochMax) ? 1u : epoch + 1u;
-                __threadfence();
-            }
+            ws_exit(p, epoch);
         }
     } else if (lane == 0) {
         // ================================================================ loader (one lane)
@@ -672,11 +927,15 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 TileInfo ti{t, 0, 0, 0};
                 if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
                 sm.info[ta.s] = ti;
+                sm.fdone[ta.s] = 0;
                 if (!valid) {
                     *reinterpret_cast<volatile int*>(&sm.end_n) = ta.k;
                     acq_done = true;
                 }
                 mbar_arrive(&sm.acq[ta.s]);
+                if constexpr (TMA && Cfg::PREFETCH) {
+                    if (valid) tma_prefetch_2d(&map_in, ti.J * TC, ti.I * TR);
+                }
 #if SAT_STATS
                 if (p.trace && valid) p.trace[8LL * t] = static_cast<long long>(globaltimer_ns());
 #endif
@@ -691,6 +950,9 @@ sat_ws_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 if (TMA && valid) {
                     mbar_arrive_expect_tx(&sm.full[sl.s], kTileBytes);
                     tma_load_2d(sm.stage[sl.s], &map_in, &sm.full[sl.s], ti.J * TC, ti.I * TR, policy);
+#if SAT_STATS
+                    if (p.trace) p.trace[8LL * ti.t + 7] = static_cast<long long>(globaltimer_ns());
+#endif
                 } else {
                     mbar_arrive(&sm.full[sl.s]);  // generic path (data read from global) or end marker
                 }

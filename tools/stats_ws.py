@@ -20,7 +20,7 @@ import satgen  # noqa: E402
 NAMES = ["tiles", "c_full_wait", "c_local", "c_walk_wait", "c_finish", "row_rounds", "col_rounds",
          "st_result_wait", "st_store", "ld_issue", "ld_empty_wait", "c_bandbar", "row_tiles", "col_tiles",
          "row_round_cyc", "col_round_cyc", "row_resolve", "col_resolve", "row_idle_rounds", "col_idle_rounds",
-         "row_load_lat", "col_load_lat", "x22", "x23"]
+         "row_load_lat", "col_load_lat", "fast_hits", "c_scan"]
 ap = argparse.ArgumentParser()
 ap.add_argument("--n", type=int, default=32768)
 ap.add_argument("--variants", default="0,1")

@@ -57,3 +57,32 @@ names = ["land-acq", "local-acq", "roww-acq", "colw-acq", "fin-acq", "store-acq"
 print(json.dumps({"variant": a.variant, "steady_tiles": len(A),
                   "median_us": {k: round(float(np.nanmedian(A[:, i]) / 1e3), 2) for i, k in enumerate(names)},
                   "p90_us": {k: round(float(np.nanpercentile(A[:, i], 90) / 1e3), 2) for i, k in enumerate(names[:13])}}))
+
+# walk wait of every interior tile: how long the compute warps sat between their local SAT and the later of
+# the two walks, split by cause: predecessor INCL not yet published at local end (chain), or published but
+# the walker had not caught it yet (poll latency)
+waits, chain, poll, diags = [], [], [], []
+for s, (I, J) in enumerate(order):
+    if I == 0 or J == 0:
+        continue
+    L, U = serial[(I, J - 1)], serial[(I - 1, J)]
+    walk = np.nanmax([T[s, ROWW], T[s, COLW]])
+    w = max(0.0, walk - T[s, LOC])
+    pred = np.nanmax([T[L, FIN], T[U, FIN]])
+    c = max(0.0, min(walk, pred) - T[s, LOC])
+    waits.append(w)
+    chain.append(c)
+    poll.append(w - c)
+    diags.append(I + J)
+waits, chain, poll, diags = map(np.array, (waits, chain, poll, diags))
+dec = np.minimum((diags * 10) // (R + C - 1), 9)
+LDI = 7
+print(json.dumps({"load_latency_us_median": round(float(np.nanmedian(T[:, LAND] - T[:, LDI])) / 1e3, 2),
+                  "load_latency_us_p90": round(float(np.nanpercentile(T[:, LAND] - T[:, LDI], 90)) / 1e3, 2),
+                  "store_after_fin_us_median": round(float(np.nanmedian(T[:, STO] - T[:, FIN])) / 1e3, 2)}))
+print(json.dumps({"mean_wait_us": round(float(np.nanmean(waits)) / 1e3, 3),
+                  "mean_chain_us": round(float(np.nanmean(chain)) / 1e3, 3),
+                  "mean_poll_us": round(float(np.nanmean(poll)) / 1e3, 3),
+                  "frac_wait_gt_0.5us": round(float(np.mean(waits > 500)), 3),
+                  "wait_by_diag_decile_us": [round(float(np.nanmean(waits[dec == q])) / 1e3, 2) for q in range(10)],
+                  "chain_by_diag_decile_us": [round(float(np.nanmean(chain[dec == q])) / 1e3, 2) for q in range(10)]}))

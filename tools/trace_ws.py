@@ -32,10 +32,10 @@ for _ in range(3):
 torch.cuda.synchronize()
 plan = sat.query_plan(1, a.n, a.n, a.n, x.data_ptr(), y.data_ptr())
 nt = plan["tiles"]
-buf = np.zeros(2 * nt, dtype=np.int64)
+buf = np.zeros(8 * nt, dtype=np.int64)
 n = ctypes.c_int64()
 _lib.check(_lib.lib().sat_debug_trace(buf.ctypes.data, nt, ctypes.byref(n)), "trace")
-acq, done = buf[0::2].astype(np.float64), buf[1::2].astype(np.float64)
+acq, done = buf[0::8].astype(np.float64), buf[6::8].astype(np.float64)  # acquired, store issued
 t0 = acq.min()
 acq -= t0
 done -= t0
