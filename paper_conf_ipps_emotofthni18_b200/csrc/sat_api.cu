@@ -151,7 +151,7 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<16, 2, 5>>(),  // 0: local SAT parked in TMEM, 2 input stages + output buffer, walkers publish
         make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 1: deferred finish, GSAT from registers
         make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch>>(),  // 2: 64 KiB tiles, 3 stages, TMA store
-        make_variant<sat::TmCfg<16, 2, 5, 1, 0>>(),  // 3: TMEM-parked, inclusive aggregates from the compute warps
+        make_variant<sat::TmCfg<16, 2, 5, 1, 2>>(),  // 3: TMEM-parked, walkers publish (blocking on the local aggregates)
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 4: classic, 32 KiB tiles, 2 stages
         make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 5: classic, 64 KiB tiles, 512 threads
     };

@@ -35,6 +35,7 @@ struct TmCfg {
     static constexpr int NT = NT_;    // tiles in flight per walker
     static constexpr bool FAST = false;
     static constexpr bool WPUB = WPUB_ != 0;  // the walkers publish the inclusive aggregates
+    static constexpr bool WPUB_WAIT = WPUB_ == 2;  // ... blocking on the tile's local aggregates
     static constexpr int RPW = TR / NW, ER = TR / 32, EC = TC / 32;
     static constexpr int NREG = RPW * 4;         // 32-bit registers per thread parked per tile
     static constexpr int TM_COLS_PER_SLOT = (NW / 4) * NREG;
@@ -60,6 +61,8 @@ struct TmSmem {
     alignas(16) V lcs[Cfg::NQ][Cfg::TC];  // local column aggregates
     alignas(8) uint64_t acq[Cfg::NQ];
     uint64_t ldone[Cfg::NQ];  // lrs / lcs written (NW arrivals)
+    int rdone[Cfg::NQ];       // k + 1 once the row walk of tile k (slot) has written rp / corner (WPUB)
+    int cdone[Cfg::NQ];       // k + 1 once the column walk of tile k has written cp
     uint64_t rowwalk[Cfg::NQ];
     uint64_t colwalk[Cfg::NQ];
     uint64_t tfree[Cfg::NQ];
@@ -407,6 +410,8 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
             mbar_init(&sm.tfree[q], 1);
             mbar_init(&sm.result[q], NW);
             mbar_init(&sm.ldone[q], NW);
+            sm.rdone[q] = 0;
+            sm.cdone[q] = 0;
         }
 #pragma unroll
         for (int s = 0; s < IN; ++s) {

@@ -106,6 +106,7 @@ struct WsCfg {
     static constexpr bool PREFETCH = (FLAGS & kWsPrefetch) != 0;
     static constexpr bool SMEM_SCAN = (FLAGS & kWsSmemScan) != 0;
     static constexpr bool WPUB = false;  // inclusive aggregates published by the compute warps
+    static constexpr bool WPUB_WAIT = false;
     static constexpr int RPW = TR / NW;   // rows per compute-warp band
     static constexpr int ER = TR / 32;    // row-vector elements per walker lane
     static constexpr int EC = TC / 32;    // column-vector elements per walker lane
@@ -205,7 +206,7 @@ __device__ __forceinline__ void ws_walker(SM& sm, const KParams<V>& p, uint32_t 
     constexpr int E = ROW ? Cfg::ER : Cfg::EC;
     constexpr int NT = Cfg::NT;
     struct Walk {
-        int active, s, I, J, pos;
+        int active, s, k, I, J, pos;
         uint32_t ph;
         uint32_t pend;
         V acc[E];
@@ -216,17 +217,57 @@ __device__ __forceinline__ void ws_walker(SM& sm, const KParams<V>& p, uint32_t 
     Walk wk[NT];
 #pragma unroll
     for (int w = 0; w < NT; ++w) wk[w].active = 0;
+    // WPUB: a resolved tile whose local aggregates were not in yet (published, and handed to the
+    // compute warps, as soon as they are; meanwhile the walker goes on with the next tiles)
+    struct Pend {
+        int on, s, k, I, J;
+        uint32_t ph;
+        V acc[E];
+        V dacc;
+    } pd;
+    pd.on = 0;
     Slot<Cfg::NQ> next;
     bool ended = false;
     int steps = 0;
     const uint64_t pol = policy_evict_last();
     constexpr int DW = 4;  // diagonal predecessors polled per round (the first is almost always inclusive)
+    // WPUB: Steps 2.A.3 / 2.B.3 (and 3.1 / 3.3 if the other walk of the tile is in) of a resolved tile
+    // whose local aggregates (lrs / lcs, kept in smem by the compute warps) are in.  The walkers are then
+    // the only publishers of inclusive aggregates: each tile's row / column words by its own walker, GS
+    // by whichever of the two publishes second (each raises its rdone / cdone flag before it looks at
+    // the other's, so at least one of them sees both).
+    auto publish = [&](int s, int k, int I, int J, const V (&acc)[E], V dacc, bool gs_only = false) {
+        if constexpr (Cfg::WPUB) {
+            const long long tidx = static_cast<long long>(I) * p.C + J;
+            V l[E];
+            uint64_t wv[E];
+#pragma unroll
+            for (int e = 0; e < E; ++e) {
+                l[e] = ROW ? sm.lrs[s][lane * E + e] : sm.lcs[s][lane * E + e];
+                wv[e] = pack(epoch, kIncl, to_bits(l[e] + acc[e]));
+            }
+            if (!gs_only && (ROW ? J > 0 : I > 0))
+                st_words_p<E>((ROW ? p.row_slots + tidx * TR : p.col_slots + tidx * TC) + lane * E, wv, pol);
+            if (lane == 31 && *reinterpret_cast<volatile int*>(ROW ? &sm.cdone[s] : &sm.rdone[s]) == k + 1) {
+                // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
+                __threadfence_block();  // acquire: the other walker's carries were written before its flag
+                const V rp1 = ROW ? acc[E - 1] : sm.rp[s][TR - 1];
+                const V cp1 = ROW ? sm.cp[s][TC - 1] : acc[E - 1];
+                const V cor = ROW ? dacc : sm.corner[s];
+                st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(cor + ((l[E - 1] + rp1) + cp1))), pol);
+            }
+        }
+    };
+    auto hand_off = [&](int s) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(ROW ? &sm.rowwalk[s] : &sm.colwalk[s]);
+    };
     while (true) {
         // ---- take newly acquired tiles into free walk slots (block only when nothing is in flight)
 #pragma unroll
         for (int w = 0; w < NT; ++w) {
             if (wk[w].active || ended) continue;
-            bool busy = false;
+            bool busy = pd.on != 0;
 #pragma unroll
             for (int v2 = 0; v2 < NT; ++v2) busy = busy || wk[v2].active;
             bool got;
@@ -246,6 +287,7 @@ __device__ __forceinline__ void ws_walker(SM& sm, const KParams<V>& p, uint32_t 
             Walk& x = wk[w];
             x.active = 1;
             x.s = next.s;
+            x.k = next.k;
             x.ph = next.ph;
             x.I = ti.I;
             x.J = ti.J;
@@ -261,7 +303,7 @@ __device__ __forceinline__ void ws_walker(SM& sm, const KParams<V>& p, uint32_t 
 #endif
             next.next();
         }
-        bool any = false;
+        bool any = pd.on != 0;
 #pragma unroll
         for (int w = 0; w < NT; ++w) any = any || wk[w].active;
         if (!any) {
@@ -352,29 +394,6 @@ __device__ __forceinline__ void ws_walker(SM& sm, const KParams<V>& p, uint32_t 
                 }
             }
             if (x.ddone && __all_sync(kFull, x.pend == 0u)) {
-                if constexpr (Cfg::WPUB) {
-                    // Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 from here, as soon as both the walk and the tile's
-                    // local aggregates (lrs / lcs, kept in smem by the compute warps) are in: successors
-                    // need not wait for the compute warps to reach the tile's Step 4.
-                    mbar_wait(&sm.ldone[x.s], x.ph);
-                    const long long tidx = static_cast<long long>(x.I) * p.C + x.J;
-                    V l[E];
-#pragma unroll
-                    for (int e = 0; e < E; ++e) l[e] = ROW ? sm.lrs[x.s][lane * E + e] : sm.lcs[x.s][lane * E + e];
-                    uint64_t wv[E];
-#pragma unroll
-                    for (int e = 0; e < E; ++e) wv[e] = pack(epoch, kIncl, to_bits(l[e] + x.acc[e]));
-                    if (ROW) {
-                        if (x.J > 0) st_words_p<E>(p.row_slots + tidx * TR + lane * E, wv, pol);
-                        mbar_wait(&sm.colwalk[x.s], x.ph);  // the column carry of the same tile
-                        if (lane == 31) {  // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
-                            const V gls = l[E - 1] + x.acc[E - 1] + sm.cp[x.s][TC - 1];
-                            st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(x.dacc + gls)), pol);
-                        }
-                    } else if (x.I > 0) {
-                        st_words_p<E>(p.col_slots + tidx * TC + lane * E, wv, pol);
-                    }
-                }
                 if (ROW) {
 #pragma unroll
                     for (int e = 0; e < E; ++e) sm.rp[x.s][lane * E + e] = x.acc[e];
@@ -384,17 +403,63 @@ __device__ __forceinline__ void ws_walker(SM& sm, const KParams<V>& p, uint32_t 
                     for (int e = 0; e < E; ++e) sm.cp[x.s][lane * E + e] = x.acc[e];
                 }
                 __syncwarp();
+                bool handed = true;
+                if constexpr (Cfg::WPUB) {
+                    // announce this half of the tile's carries to the other walker (for GS), then publish
+                    // now if the local aggregates are in, else park the tile and go on walking
+                    if (lane == 0) {
+                        *reinterpret_cast<volatile int*>(ROW ? &sm.rdone[x.s] : &sm.cdone[x.s]) = x.k + 1;
+                        __threadfence_block();
+                    }
+                    __syncwarp();
+                    if (pd.on) {  // rare: two tiles waiting for their local aggregates
+                        mbar_wait(&sm.ldone[pd.s], pd.ph);
+                        publish(pd.s, pd.k, pd.I, pd.J, pd.acc, pd.dacc);
+                        hand_off(pd.s);
+                        pd.on = 0;
+                    }
+                    if (Cfg::WPUB_WAIT) {
+                        mbar_wait(&sm.ldone[x.s], x.ph);
+                        publish(x.s, x.k, x.I, x.J, x.acc, x.dacc);
+                        if (ROW && __shfl_sync(kFull, *reinterpret_cast<volatile int*>(&sm.cdone[x.s]) != x.k + 1, 31)) {
+                            // GS needs the column carry too: wait for the column walker, then publish it
+                            mbar_wait(&sm.colwalk[x.s], x.ph);
+                            publish(x.s, x.k, x.I, x.J, x.acc, x.dacc, true);
+                        }
+                    } else if (__shfl_sync(kFull, static_cast<int>(mbar_test(&sm.ldone[x.s], x.ph)), 0)) {
+                        publish(x.s, x.k, x.I, x.J, x.acc, x.dacc);
+                    } else {
+                        pd.on = 1;
+                        pd.s = x.s;
+                        pd.k = x.k;
+                        pd.I = x.I;
+                        pd.J = x.J;
+                        pd.ph = x.ph;
+#pragma unroll
+                        for (int e = 0; e < E; ++e) pd.acc[e] = x.acc[e];
+                        pd.dacc = x.dacc;
+                        handed = false;
+                    }
+                }
                 if (lane == 0) {
 #if SAT_STATS
                     if (p.trace) p.trace[8LL * sm.info[x.s].t + (ROW ? 3 : 4)] = static_cast<long long>(globaltimer_ns());
 #endif
-                    mbar_arrive(ROW ? &sm.rowwalk[x.s] : &sm.colwalk[x.s]);
                     WS_ST(ROW ? kWsRowTiles : kWsColTiles, 1);
 #if SAT_STATS
                     WS_ST(ROW ? kWsRowResolve : kWsColResolve, clock64() - x.t_acq);
 #endif
                 }
+                if (handed) hand_off(x.s);
                 x.active = 0;
+                progress = true;
+            }
+        }
+        if constexpr (Cfg::WPUB) {
+            if (pd.on && __shfl_sync(kFull, static_cast<int>(mbar_test(&sm.ldone[pd.s], pd.ph)), 0)) {
+                publish(pd.s, pd.k, pd.I, pd.J, pd.acc, pd.dacc);
+                hand_off(pd.s);
+                pd.on = 0;
                 progress = true;
             }
         }
