@@ -26,7 +26,7 @@
 
 namespace sat {
 
-template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1>
+template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2>
 struct TmCfg {
     static constexpr int TR = 128, TC = 128, NW = NW_;
     static constexpr int IN = IN_;    // input stages
@@ -38,15 +38,16 @@ struct TmCfg {
     static constexpr bool WPUB_WAIT = WPUB_ == 2;  // ... blocking on the tile's local aggregates
     static constexpr int RPW = TR / NW, ER = TR / 32, EC = TC / 32;
     static constexpr int NREG = RPW * 4;         // 32-bit registers per thread parked per tile
+    static constexpr int D = D_;                 // TMEM parking depth: finish(k) runs after local(k + D - 1)
     static constexpr int TM_COLS_PER_SLOT = (NW / 4) * NREG;
-    static constexpr int TM_COLS = 2 * TM_COLS_PER_SLOT <= 32 ? 32 : 2 * TM_COLS_PER_SLOT <= 64 ? 64
-                                 : 2 * TM_COLS_PER_SLOT <= 128 ? 128 : 2 * TM_COLS_PER_SLOT <= 256 ? 256 : 512;
+    static constexpr int TM_COLS = D * TM_COLS_PER_SLOT <= 32 ? 32 : D * TM_COLS_PER_SLOT <= 64 ? 64
+                                 : D * TM_COLS_PER_SLOT <= 128 ? 128 : D * TM_COLS_PER_SLOT <= 256 ? 256 : 512;
     static constexpr int ROW_WARP = NW, COL_WARP = NW + 1, STORE_WARP = NW + 2, LOAD_WARP = NW + 3;
     static constexpr int THREADS = (NW + 4) * 32;
     static_assert(NW % 4 == 0 && TR % NW == 0 && RPW % 4 == 0, "compute warps cover the 4 TMEM lane quarters");
     static_assert(NREG == 16 || NREG == 32, "tcgen05 32x32b.x16 / .x32 parking");
-    static_assert(2 * TM_COLS_PER_SLOT <= 512, "TMEM columns");
-    static_assert(IN >= 1 && NQ >= IN + 1 && NQ <= 16, "rings");
+    static_assert(D >= 2 && D * TM_COLS_PER_SLOT <= 512, "TMEM columns");
+    static_assert(IN >= 1 && NQ >= IN + D - 1 && NQ <= 16, "rings");
 };
 
 template <typename V, typename Cfg>
@@ -149,7 +150,7 @@ __device__ __forceinline__ uint32_t tm_addr(uint32_t base, int warp, int slot) {
 }
 
 // Step 1 + local SAT + Steps 2.A.1 / 2.B.1 of tile k (input stage sl, tile slot tq); parks the block in
-// TMEM slot k & 1.  Returns false at the end marker.
+// TMEM slot k % D.  Returns false at the end marker.
 template <typename V, typename Cfg, bool TMA>
 __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p, const Slot<Cfg::IN>& sl,
                                          const Slot<Cfg::NQ>& tq, uint32_t epoch, int warp, int lane) {
@@ -274,7 +275,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p
     for (int r = 0; r < RPW; ++r)
 #pragma unroll
         for (int c = 0; c < 4; ++c) r32[r * 4 + c] = to_bits(v[r][c]);
-    tmem_st<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k & 1), r32);
+    tmem_st<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k % Cfg::D), r32);
     SAT_CLK(c2);
     if (warp == 0 && lane == 0) WS_ST(kWsLocal, c2 - c1);
 #if SAT_STATS
@@ -284,7 +285,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p
 }
 
 // Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 and Step 4 of tile k (tile slot tq; its block parked in TMEM slot
-// k & 1), GSAT into the output buffer (use number `ou` of it).
+// k % D), GSAT into the output buffer (use number `ou` of it).
 template <typename V, typename Cfg, bool TMA, bool CARRY>
 __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& p, const Slot<Cfg::NQ>& tq,
                                           uint32_t ou, uint32_t epoch, int warp, int lane) {
@@ -298,7 +299,7 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& 
     V v[RPW][4];
     {
         uint32_t r32[Cfg::NREG];
-        tmem_ld<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k & 1), r32);
+        tmem_ld<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k % Cfg::D), r32);
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
 #pragma unroll
@@ -428,24 +429,28 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
 
     if (warp < NW) {
         // ================================================================ compute warps
-        // local(0), then {local(k+1), finish(k)}: the walks of tile k run during local(k+1)
+        // local(0 .. D-2), then {local(k+D-1), finish(k)}: the walks of tile k run during the D-1 locals
+        // that follow it
         Slot<IN> sl;
-        Slot<Cfg::NQ> tq;
+        Slot<Cfg::NQ> tql, tqf;
         uint32_t ou = 0;  // uses of the output buffer so far
-        bool have = tm_local<V, Cfg, TMA>(sm, p, sl, tq, epoch, warp, lane);
-        while (have) {
-            Slot<IN> sl2 = sl;
-            Slot<Cfg::NQ> tq2 = tq;
-            sl2.next();
-            tq2.next();
-            const bool have2 = tm_local<V, Cfg, TMA>(sm, p, sl2, tq2, epoch, warp, lane);
-            const TileInfo ti = sm.info[tq.s];
+        int parked = 0;
+        bool more = true;
+        while (more && parked < Cfg::D - 1) {
+            more = tm_local<V, Cfg, TMA>(sm, p, sl, tql, epoch, warp, lane);
+            if (more) { ++parked; sl.next(); tql.next(); }
+        }
+        while (parked > 0) {
+            if (more) {
+                more = tm_local<V, Cfg, TMA>(sm, p, sl, tql, epoch, warp, lane);
+                if (more) { ++parked; sl.next(); tql.next(); }
+            }
+            const TileInfo ti = sm.info[tqf.s];
             const bool ragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
-            tm_finish<V, Cfg, TMA, CARRY>(sm, p, tq, ou, epoch, warp, lane);
+            tm_finish<V, Cfg, TMA, CARRY>(sm, p, tqf, ou, epoch, warp, lane);
             if (!ragged) ++ou;
-            sl = sl2;
-            tq = tq2;
-            have = have2;
+            tqf.next();
+            --parked;
         }
         tc_fence_before();
         named_bar_sync(2, NW * 32);
