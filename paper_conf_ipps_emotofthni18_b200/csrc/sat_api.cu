@@ -94,9 +94,9 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
 };
 
-template <int NW, int IN, int NQ, int NT, int WPUB, int D>
-struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D>> {
-    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D>;
+template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT>;
     static constexpr int threads = Cfg::THREADS;
     static constexpr int family = 2;
     template <typename V>
@@ -154,10 +154,10 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<16, 2, 5, 1, 2>>(),  // 3: TMEM-parked, walkers publish (blocking on the local aggregates)
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 4: classic, 32 KiB tiles, 2 stages
         make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 5: classic, 64 KiB tiles, 512 threads
-        make_variant<sat::TmCfg<16, 2, 5, 1, 1, 3>>(),  // 6: experimental
-        make_variant<sat::TmCfg<16, 2, 6, 1, 1, 3>>(),  // 7
-        make_variant<sat::TmCfg<16, 2, 7, 1, 1, 4>>(),  // 8
-        make_variant<sat::TmCfg<16, 2, 8, 1, 1, 4>>(),  // 9
+        make_variant<sat::TmCfg<16, 2, 7, 1, 1, 4>>(),  // 6: experimental
+        make_variant<sat::TmCfg<16, 3, 8, 1, 3, 4, 1>>(),  // 7
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 8
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),  // 9
     };
     return vs;
 }

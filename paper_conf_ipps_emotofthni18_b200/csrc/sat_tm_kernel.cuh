@@ -26,7 +26,7 @@
 
 namespace sat {
 
-template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2>
+template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0>
 struct TmCfg {
     static constexpr int TR = 128, TC = 128, NW = NW_;
     static constexpr int IN = IN_;    // input stages
@@ -36,9 +36,11 @@ struct TmCfg {
     static constexpr bool FAST = false;
     static constexpr bool WPUB = WPUB_ != 0;  // the walkers publish the inclusive aggregates
     static constexpr bool WPUB_WAIT = WPUB_ == 2;  // ... blocking on the tile's local aggregates
+    static constexpr bool DECOUPLED = WPUB_ == 3;  // tm_walker: GLS published as a local corner word
     static constexpr int RPW = TR / NW, ER = TR / 32, EC = TC / 32;
     static constexpr int NREG = RPW * 4;         // 32-bit registers per thread parked per tile
     static constexpr int D = D_;                 // TMEM parking depth: finish(k) runs after local(k + D - 1)
+    static constexpr bool DIRECT = DIRECT_ != 0; // GSAT stored from registers (st.global.cs), no output buffer
     static constexpr int TM_COLS_PER_SLOT = (NW / 4) * NREG;
     static constexpr int TM_COLS = D * TM_COLS_PER_SLOT <= 32 ? 32 : D * TM_COLS_PER_SLOT <= 64 ? 64
                                  : D * TM_COLS_PER_SLOT <= 128 ? 128 : D * TM_COLS_PER_SLOT <= 256 ? 256 : 512;
@@ -53,7 +55,7 @@ struct TmCfg {
 template <typename V, typename Cfg>
 struct TmSmem {
     alignas(1024) V stage[Cfg::IN][Cfg::TR * Cfg::TC];  // input ring (TMA loads)
-    alignas(1024) V out[Cfg::TR * Cfg::TC];             // GSAT of one tile (TMA store source)
+    alignas(1024) V out[Cfg::DIRECT ? 4 : Cfg::TR * Cfg::TC];  // GSAT of one tile (TMA store source)
     alignas(16) V band[2][Cfg::NW][Cfg::TC];
     alignas(16) V rp[Cfg::NQ][Cfg::TR];
     alignas(16) V cp[Cfg::NQ][Cfg::TC];
@@ -64,6 +66,8 @@ struct TmSmem {
     uint64_t ldone[Cfg::NQ];  // lrs / lcs written (NW arrivals)
     int rdone[Cfg::NQ];       // k + 1 once the row walk of tile k (slot) has written rp / corner (WPUB)
     int cdone[Cfg::NQ];       // k + 1 once the column walk of tile k has written cp
+    int rres[Cfg::NQ];        // DECOUPLED: k + 1 once the row walk of tile k has written rp (corner maybe not)
+    int lw[Cfg::NQ][Cfg::NW]; // DECOUPLED: k + 1 once compute warp w has written its lrs (and lcs) of tile k
     uint64_t rowwalk[Cfg::NQ];
     uint64_t colwalk[Cfg::NQ];
     uint64_t tfree[Cfg::NQ];
@@ -268,6 +272,39 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p
                 to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
         __syncwarp();
         if (lane == 0) mbar_arrive(&sm.ldone[tq.s]);
+        if constexpr (Cfg::DECOUPLED) {
+            // whoever comes last publishes (see tm_walker): raise this warp's flag, then look at the walkers'
+            __threadfence_block();
+            if (lane == 0) *reinterpret_cast<volatile int*>(&sm.lw[tq.s][warp]) = tq.k + 1;
+            __threadfence_block();
+            if (lane == 31 && J > 0 && *reinterpret_cast<volatile int*>(&sm.rres[tq.s]) == tq.k + 1) {
+                __threadfence_block();
+                uint64_t* rs = p.row_slots + tidx * TR + row0;
+#pragma unroll
+                for (int r = 0; r < RPW; r += 2)
+                    st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + sm.rp[tq.s][row0 + r])),
+                                  pack(epoch, kIncl, to_bits(v[r + 1][3] + sm.rp[tq.s][row0 + r + 1])), pol);
+            }
+            if (warp == NW - 1) {
+                const int cd = __shfl_sync(kFull, *reinterpret_cast<volatile int*>(&sm.cdone[tq.s]), 0);
+                if (cd == tq.k + 1) {
+                    __threadfence_block();
+                    if (I > 0) {
+                        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[tq.s][col0]);
+                        uint64_t* cs = p.col_slots + tidx * TC + col0;
+                        st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + from_bits<V>(c4.x))),
+                                      pack(epoch, kIncl, to_bits(v[RPW - 1][1] + from_bits<V>(c4.y))), pol);
+                        st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + from_bits<V>(c4.z))),
+                                      pack(epoch, kIncl, to_bits(v[RPW - 1][3] + from_bits<V>(c4.w))), pol);
+                    }
+                    if (lane == 31 && *reinterpret_cast<volatile int*>(&sm.rdone[tq.s]) == tq.k + 1) {
+                        __threadfence_block();
+                        const V gs = sm.corner[tq.s] + ((v[RPW - 1][3] + sm.rp[tq.s][TR - 1]) + sm.cp[tq.s][TC - 1]);
+                        st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(gs)), pol);
+                    }
+                }
+            }
+        }
     }
     // park the block
     uint32_t r32[Cfg::NREG];
@@ -359,7 +396,18 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& 
 #pragma unroll
         for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + (rt[r] + colterm[c]);
     const bool ragged = !TMA || ((J == p.C - 1) && (p.cols & 3) != 0);
-    if (!ragged) {
+    if (Cfg::DIRECT && !ragged) {
+        // Step 4 store straight from registers: a lane writes 16 contiguous bytes of each of its rows
+        // (a warp row = 512 contiguous bytes); columns >= cols are clipped, rows >= rows skipped
+        const long long gj = static_cast<long long>(J) * TC + col0;
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const long long gi = static_cast<long long>(I) * TR + row0 + r;
+            if (gi < p.rows && gj < p.cols)
+                __stcs(reinterpret_cast<uint4*>(p.dst + gi * p.pitch + gj),
+                       make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3])));
+        }
+    } else if (!ragged) {
         mbar_wait(&sm.ofree, (ou & 1u) ^ 1u);  // the previous tile's store has read `out`
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
@@ -384,6 +432,146 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& 
     if (lane == 0) mbar_arrive(&sm.result[q]);
     SAT_CLK(c2);
     if (warp == 0 && lane == 0) WS_ST(kWsFinish, c2 - c1);
+}
+
+// Walker with a decoupled diagonal look-back (Cfg::DECOUPLED), one tile at a time, in acquisition order.
+//
+// Row walker: row look-back (Step 2.A.2) and diagonal look-back (Step 3.2).  Column
+// walker: column look-back (Step 2.B.2).  A walker never waits for anything but the words it polls: it
+// hands a tile's carries to the compute warps (smem + rowwalk / colwalk) and goes on with the next tile.
+// The inclusive words need the local aggregates too, so they are published by whichever side comes
+// last, each raising its flag before it looks at the other's:
+//   row words (Step 2.A.3)  compute warp w (flag lw[w], its RPW rows)   vs the row walker (rres)
+//   column words (2.B.3)    compute warp NW-1 (lw[NW-1])                 vs the column walker (cdone)
+//   GS (Step 3.3)           compute warp NW-1, column walker, row walker (rdone: rp and the corner)
+// Both sides compute the same sums from the same operands, so a double publication writes equal bits.
+// The corner word goes through two states like the vector words: while its diagonal look-back is
+// still open, the row walker publishes GLS(I,J) = total + rp[TR-1] + cp[TC-1] (Step 3.1)
+// with kind "local"; GS(I,J) = GS(I-1,J-1) + GLS(I,J) follows with kind "inclusive" (only after rdone,
+// which the row walker raises after any GLS store; should another warp's GS store still land first,
+// the word merely reads "local" again: readers then walk one tile further, and the edge tiles, whose
+// walk is empty, only ever publish GS).  A diagonal look-back therefore sums GLS words up to
+// the first GS word (reading R8) instead of waiting for GS(I-1,J-1): no chain in any of the
+// three directions waits for a neighbour's completion.
+template <typename V, typename Cfg, bool ROW>
+__device__ __forceinline__ void tm_walker(TmSmem<V, Cfg>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, RPW = Cfg::RPW, NW = Cfg::NW;
+    constexpr int E = ROW ? Cfg::ER : Cfg::EC;
+    constexpr int DW = 4;  // diagonal predecessors polled per round
+    const uint64_t pol = policy_evict_last();
+    auto flag = [&](const int* f) { return *reinterpret_cast<const volatile int*>(f); };
+    for (Slot<Cfg::NQ> nx;; nx.next()) {
+        if (!wait_acquired(sm, nx.s, nx.ph, nx.k)) break;
+        const TileInfo ti = sm.info[nx.s];
+        if (ti.t >= p.ntiles) break;
+        const int s = nx.s, k = nx.k, I = ti.I, J = ti.J;
+        const long long tidx = static_cast<long long>(I) * p.C + J;
+        const long long step = ROW ? static_cast<long long>(TR) : static_cast<long long>(p.C) * TC;
+        uint64_t* const own = ROW ? p.row_slots + tidx * TR : p.col_slots + tidx * TC;
+        int pos = ROW ? J - 1 : I - 1;
+        uint32_t pend = pos >= 0 ? (1u << E) - 1u : 0u;
+        V acc[E];
+#pragma unroll
+        for (int e = 0; e < E; ++e) acc[e] = V(0);
+        bool ddone = ROW ? (I == 0 || J == 0) : true;
+        V dacc = V(0);
+        int dbase = 1;
+        bool cin = false, lpub = false;
+        while (true) {
+            // ---- issue this round's loads
+            uint64_t w0[E], w1[E], wd = 0;
+            const bool have1 = pos >= 1;
+            if (pend) {
+                const uint64_t* q = own - (ROW ? static_cast<long long>(J - pos) * TR
+                                               : static_cast<long long>(I - pos) * p.C * TC) + lane * E;
+                ld_words_p<E>(q, w0, pol);
+                if (have1) ld_words_p<E>(q - step, w1, pol);
+            }
+            const int kk = dbase + lane;
+            const bool dinr = ROW && !ddone && lane < DW && (I - kk >= 0) && (J - kk >= 0);
+            if (dinr) wd = ld_relaxed_p(p.corner_slots + static_cast<long long>(I - kk) * p.C + (J - kk), pol);
+            // ---- consume
+            bool progress = false;
+            if (pend) progress = lb_consume<V, E>(pend, pos, acc, w0, w1, have1, epoch);
+            if (ROW && !ddone) {
+                const bool ready = !dinr || word_ready(wd, epoch);
+                const unsigned incl = __ballot_sync(kFull, dinr && ready && word_kind(wd) == kIncl);
+                const unsigned notready = __ballot_sync(kFull, !ready);
+                const int f = incl ? (__ffs(incl) - 1) : DW;
+                const unsigned need = (2u << (f < DW ? f : DW - 1)) - 1u;
+                if (!(notready & need)) {
+                    V val = (dinr && lane <= f) ? from_bits<V>(static_cast<uint32_t>(wd)) : V(0);
+#pragma unroll
+                    for (int d = DW / 2; d >= 1; d >>= 1) val = val + __shfl_xor_sync(kFull, val, d);
+                    dacc = dacc + __shfl_sync(kFull, val, 0);
+                    if (f < DW) ddone = true; else dbase += DW;
+                    progress = true;
+                }
+            }
+            if (!cin && __all_sync(kFull, pend == 0u)) {
+                // carries -> smem, raise the flag, then publish the inclusive words of the rows / columns
+                // whose local aggregates are already in
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    if (ROW) sm.rp[s][lane * E + e] = acc[e];
+                    else sm.cp[s][lane * E + e] = acc[e];
+                }
+                __syncwarp();
+                __threadfence_block();
+                if (lane == 0) *reinterpret_cast<volatile int*>(ROW ? &sm.rres[s] : &sm.cdone[s]) = k + 1;
+                __threadfence_block();
+                const int owner = ROW ? (lane * E) / RPW : NW - 1;  // compute warp holding these locals
+                if ((ROW ? J > 0 : I > 0) && flag(&sm.lw[s][owner]) == k + 1) {
+                    __threadfence_block();
+                    uint64_t wv[E];
+#pragma unroll
+                    for (int e = 0; e < E; ++e) {
+                        const V l = ROW ? sm.lrs[s][lane * E + e] : sm.lcs[s][lane * E + e];
+                        wv[e] = pack(epoch, kIncl, to_bits(l + acc[e]));
+                    }
+                    st_words_p<E>(own + lane * E, wv, pol);
+                }
+                cin = true;
+                progress = true;
+            }
+            if (ROW && cin && !ddone && !lpub) {  // Step 3.1: GLS, published as a local corner word
+                int go = 0;
+                if (lane == 31 && flag(&sm.cdone[s]) == k + 1 && flag(&sm.lw[s][NW - 1]) == k + 1) {
+                    __threadfence_block();
+                    const V gls = (sm.lrs[s][TR - 1] + acc[E - 1]) + sm.cp[s][TC - 1];
+                    st_relaxed_p(p.corner_slots + tidx, pack(epoch, kLocal, to_bits(gls)), pol);
+                    go = 1;
+                }
+                lpub = __shfl_sync(kFull, go, 31) != 0;
+            }
+            if (cin && ddone) break;
+            if (!progress) __nanosleep(32);
+        }
+        // ---- Step 3.3 (GS, by whoever comes last) and the hand-off
+        if (ROW) {
+            if (lane == 0) sm.corner[s] = dacc;
+            __syncwarp();
+            __threadfence_block();
+            if (lane == 0) *reinterpret_cast<volatile int*>(&sm.rdone[s]) = k + 1;
+            __threadfence_block();
+            if (lane == 31 && flag(&sm.cdone[s]) == k + 1 && flag(&sm.lw[s][NW - 1]) == k + 1) {
+                __threadfence_block();
+                const V gs = dacc + ((sm.lrs[s][TR - 1] + acc[E - 1]) + sm.cp[s][TC - 1]);
+                st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(gs)), pol);
+            }
+        } else {
+            if (lane == 31 && flag(&sm.rdone[s]) == k + 1 && flag(&sm.lw[s][NW - 1]) == k + 1) {
+                __threadfence_block();
+                const V gs = sm.corner[s] + ((sm.lrs[s][TR - 1] + sm.rp[s][TR - 1]) + acc[E - 1]);
+                st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(gs)), pol);
+            }
+        }
+#if SAT_STATS
+        if (p.trace && lane == 0) p.trace[8LL * ti.t + (ROW ? 3 : 4)] = static_cast<long long>(globaltimer_ns());
+#endif
+        __syncwarp();
+        if (lane == 0) mbar_arrive(ROW ? &sm.rowwalk[s] : &sm.colwalk[s]);
+    }
 }
 
 template <typename V, typename Cfg, bool TMA, bool CARRY>
@@ -413,6 +601,8 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
             mbar_init(&sm.ldone[q], NW);
             sm.rdone[q] = 0;
             sm.cdone[q] = 0;
+            sm.rres[q] = 0;
+            for (int w = 0; w < NW; ++w) sm.lw[q][w] = 0;
         }
 #pragma unroll
         for (int s = 0; s < IN; ++s) {
@@ -456,9 +646,11 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         named_bar_sync(2, NW * 32);
         if (warp == 0) tmem_dealloc(sm.tmem_base, Cfg::TM_COLS);
     } else if (warp == Cfg::ROW_WARP) {
-        ws_walker<V, Cfg, true>(sm, p, epoch, lane);
+        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, true>(sm, p, epoch, lane);
+        else ws_walker<V, Cfg, true>(sm, p, epoch, lane);
     } else if (warp == Cfg::COL_WARP) {
-        ws_walker<V, Cfg, false>(sm, p, epoch, lane);
+        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, false>(sm, p, epoch, lane);
+        else ws_walker<V, Cfg, false>(sm, p, epoch, lane);
     } else if (warp == Cfg::STORE_WARP) {
         // ================================================================ storer (one lane)
         if (lane == 0) {
@@ -476,7 +668,7 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 SAT_CLK(u1);
                 WS_ST(kWsStResultWait, u1 - u0);
                 const bool ragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
-                if (!ragged) {
+                if (!Cfg::DIRECT && !ragged) {
                     tma_store_2d_hint(&map_out, sm.out, ti.J * TC, ti.I * TR, spol);
                     bulk_commit();
 #if SAT_STATS

@@ -105,7 +105,7 @@ def test_int32_bit_exact(sat, shape):
     assert_i32_exact(run_sat(sat, a), a)
 
 
-@pytest.mark.parametrize("variant", range(6))
+@pytest.mark.parametrize("variant", range(12))
 @pytest.mark.parametrize("order", [0, 1])
 def test_int32_every_variant_and_order(sat, variant, order):
     if variant >= sat.num_variants():

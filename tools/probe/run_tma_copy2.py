@@ -19,7 +19,7 @@ for _ in range(10):
 e1.record()
 torch.cuda.synchronize()
 print(f"torch copy_: {e0.elapsed_time(e1) / 10:.4f} ms", flush=True)
-CFGS = [(128, 128, 2), (64, 256, 2), (32, 512, 2)] if len(sys.argv) > 4 else [(128, 128, 2), (64, 256, 2), (32, 512, 2), (16, 1024, 2), (128, 128, 3), (64, 256, 3), (32, 512, 3),
+CFGS = [(128, 128, 2), (128, 128, 3), (64, 256, 3), (32, 512, 3)] if len(sys.argv) > 4 else [(128, 128, 2), (64, 256, 2), (32, 512, 2), (16, 1024, 2), (128, 128, 3), (64, 256, 3), (32, 512, 3),
         (16, 1024, 3), (32, 256, 4), (32, 256, 6), (16, 512, 4), (16, 512, 6), (64, 512, 1), (32, 1024, 1),
         (32, 1024, 2), (16, 2048, 2), (32, 128, 4), (64, 128, 4)]
 modes = [int(m) for m in (sys.argv[2] if len(sys.argv) > 2 else "0,1").split(",")]

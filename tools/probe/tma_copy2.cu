@@ -108,7 +108,7 @@ template <int TR, int TC, int ST, int MODE>
 __global__ void __launch_bounds__((NW + 2) * 32, 1) copy_kernel(const __grid_constant__ CUtensorMap mi,
                                                                  const __grid_constant__ CUtensorMap mo, int R, int C,
                                                                  int order, unsigned int* counter,
-                                                                 unsigned long long* lat) {
+                                                                 unsigned long long* lat, float* dst, int n) {
     extern __shared__ __align__(1024) unsigned char raw[];
     float* stage = reinterpret_cast<float*>(raw);
     constexpr int NO = (ST + 2) * TR * TC * 4 <= 227 * 1024 ? 2 : 1;
@@ -120,7 +120,7 @@ __global__ void __launch_bounds__((NW + 2) * 32, 1) copy_kernel(const __grid_con
     constexpr uint32_t kBytes = TR * TC * 4;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (threadIdx.x == 0) {
-        for (int s = 0; s < ST; ++s) { minit(&full[s], 1); minit(&empty[s], MODE == 1 ? NW : 1); }
+        for (int s = 0; s < ST; ++s) { minit(&full[s], 1); minit(&empty[s], MODE >= 1 ? NW : 1); }
         for (int s = 0; s < 2; ++s) { minit(&ofull[s], NW); minit(&ofree[s], 1); }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
@@ -145,7 +145,7 @@ __global__ void __launch_bounds__((NW + 2) * 32, 1) copy_kernel(const __grid_con
             (void)sum; (void)cnt;
         }
     } else if (warp == NW + 1) {
-        if (lane == 0) {  // storer
+        if (MODE != 2 && lane == 0) {  // storer
             unsigned long long sum = 0, cnt = 0;
             for (int k = 0;; ++k) {
                 const int s = k % ST;
@@ -178,7 +178,7 @@ __global__ void __launch_bounds__((NW + 2) * 32, 1) copy_kernel(const __grid_con
             atomicAdd(&lat[0], sum);
             atomicAdd(&lat[1], cnt);
         }
-    } else if (MODE == 1) {
+    } else if (MODE >= 1) {
         // compute warps: stage -> registers -> out
         constexpr int RPW = TR / NW > 0 ? TR / NW : 1;
         constexpr int V4 = TC / 128;  // float4 per lane per row
@@ -188,6 +188,7 @@ __global__ void __launch_bounds__((NW + 2) * 32, 1) copy_kernel(const __grid_con
             const int t = tid_of[s];
             const int o = k % NO;
             if (t >= ntiles) {
+                if (MODE == 2) break;
                 if (k >= NO) mwait(&ofree[o], ((k / NO) & 1) ^ 1);
                 if (warp == 0 && lane == 0) otid[o] = t;
                 __syncwarp();
@@ -203,6 +204,19 @@ __global__ void __launch_bounds__((NW + 2) * 32, 1) copy_kernel(const __grid_con
                     v[r][u] = *reinterpret_cast<const float4*>(&st[(warp * RPW + r) * TC + u * 128 + lane * 4]);
             __syncwarp();
             if (lane == 0) marrive(&empty[s]);
+            if constexpr (MODE == 2) {
+                int I, J;
+                tile_ij(t, R, C, order, I, J);
+#pragma unroll
+                for (int r = 0; r < RPW; ++r)
+#pragma unroll
+                    for (int u = 0; u < V4; ++u) {
+                        float4* g = reinterpret_cast<float4*>(dst + static_cast<long long>(I * TR + warp * RPW + r) * n +
+                                                              J * TC + u * 128 + lane * 4);
+                        __stcs(g, v[r][u]);
+                    }
+                continue;
+            }
             if (k >= NO) mwait(&ofree[o], ((k / NO) & 1) ^ 1);
             if (warp == 0 && lane == 0) otid[o] = t;
             float* ob = out + o * TR * TC;
@@ -265,10 +279,10 @@ int run(const float* src, float* dst, int n, int ctas, int reps, int order, int 
     cudaEvent_t e0, e1;
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);
-    for (int w = 0; w < 2; ++w) k<<<ctas, (NW + 2) * 32, smem>>>(mi, mo, n / TR, n / TC, order, ctr + reps + w, lat);
+    for (int w = 0; w < 2; ++w) k<<<ctas, (NW + 2) * 32, smem>>>(mi, mo, n / TR, n / TC, order, ctr + reps + w, lat, dst, n);
     cudaMemset(lat, 0, 16);
     cudaEventRecord(e0);
-    for (int r = 0; r < reps; ++r) k<<<ctas, (NW + 2) * 32, smem>>>(mi, mo, n / TR, n / TC, order, ctr + r, lat);
+    for (int r = 0; r < reps; ++r) k<<<ctas, (NW + 2) * 32, smem>>>(mi, mo, n / TR, n / TC, order, ctr + r, lat, dst, n);
     cudaEventRecord(e1);
     cudaEventSynchronize(e1);
     cudaEventElapsedTime(ms, e0, e1);
@@ -288,7 +302,7 @@ extern "C" int tma_copy2(const float* src, float* dst, int n, int tr, int tc, in
                          int order, int promo, float* ms, double* lat_cyc) {
 #define CASE(A, B, C, M) \
     if (tr == A && tc == B && stages == C && mode == M) return run<A, B, C, M>(src, dst, n, ctas, reps, order, promo, ms, lat_cyc);
-#define CASES(A, B, C) CASE(A, B, C, 0) CASE(A, B, C, 1)
+#define CASES(A, B, C) CASE(A, B, C, 0) CASE(A, B, C, 1) CASE(A, B, C, 2)
     CASES(128, 128, 2) CASES(128, 128, 3) CASES(64, 256, 2) CASES(64, 256, 3) CASES(32, 512, 2) CASES(32, 512, 3)
     CASES(16, 1024, 2) CASES(16, 1024, 3) CASES(32, 256, 4) CASES(32, 256, 6) CASES(16, 512, 4) CASES(16, 512, 6)
     CASES(64, 512, 1) CASES(32, 1024, 1) CASES(32, 1024, 2) CASES(16, 2048, 2) CASES(32, 128, 4) CASES(64, 128, 4)
