@@ -798,7 +798,11 @@ SAT_API sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t col
 SAT_API sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm) {
     if (variant < -1 || variant >= static_cast<int>(variants().size()))
         return fail(SAT_ERR_INVALID_VALUE, "unknown variant %d", variant);
+#if SAT_STATS
+    if (order < 0 || (order & 15) > 1) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
+#else
     if (order < 0 || order > 1) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
+#endif
     if (ctas_per_sm < 0) return fail(SAT_ERR_INVALID_VALUE, "ctas_per_sm < 0");
     std::lock_guard<std::mutex> lk(g_mu);
     g_variant = variant;

@@ -99,7 +99,7 @@ __device__ __forceinline__ long long tri_floor_inv(long long s) {  // largest k 
 }
 
 __device__ __forceinline__ void tile_of_serial(int s_, int R, int C, int order, int& I, int& J) {
-    if (order == 1) {
+    if ((order & 15) == 1) {
         I = s_ / C;
         J = s_ - I * C;
         return;

@@ -108,7 +108,6 @@ __device__ __forceinline__ void tmem_st<32>(uint32_t taddr, const uint32_t (&r)[
         "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]),
         "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31])
         : "memory");
-    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }
 template <>
 __device__ __forceinline__ void tmem_st<16>(uint32_t taddr, const uint32_t (&r)[16]) {
@@ -118,8 +117,10 @@ __device__ __forceinline__ void tmem_st<16>(uint32_t taddr, const uint32_t (&r)[
         "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
         "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
         : "memory");
-    asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
 }
+// tcgen05.st is asynchronous: completion is awaited (tmem_st_wait) only before the block is read back
+// (the source registers are consumed at issue)
+__device__ __forceinline__ void tmem_st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void tmem_ld(uint32_t taddr, uint32_t (&r)[N]);
 template <>
@@ -223,22 +224,14 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p
     *reinterpret_cast<uint4*>(&sm.band[par][warp][col0]) =
         make_uint4(to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
     named_bar_sync(1, NW * 32);
-    {
-        const int tid = warp * 32 + lane;
-        if (tid < TC) {
-            V b[NW];
-#pragma unroll
-            for (int u = 0; u < NW; ++u) b[u] = sm.band[par][u][tid];
-            V run = V(0);
-#pragma unroll
-            for (int u = 0; u < NW; ++u) {
-                sm.band[par][u][tid] = run;
-                run = run + b[u];
-            }
+    {   // band offsets: warp w adds the bottoms of bands 0 .. w-1 (one barrier, no serial scan)
+        V off[4] = {V(0), V(0), V(0), V(0)};
+#pragma unroll 4
+        for (int u = 0; u < warp; ++u) {
+            const uint4 q = *reinterpret_cast<const uint4*>(&sm.band[par][u][col0]);
+            off[0] = off[0] + from_bits<V>(q.x); off[1] = off[1] + from_bits<V>(q.y);
+            off[2] = off[2] + from_bits<V>(q.z); off[3] = off[3] + from_bits<V>(q.w);
         }
-        named_bar_sync(1, NW * 32);
-        const uint4 q = *reinterpret_cast<const uint4*>(&sm.band[par][warp][col0]);
-        const V off[4] = {from_bits<V>(q.x), from_bits<V>(q.y), from_bits<V>(q.z), from_bits<V>(q.w)};
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
 #pragma unroll
@@ -336,6 +329,7 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& 
     V v[RPW][4];
     {
         uint32_t r32[Cfg::NREG];
+        tmem_st_wait();
         tmem_ld<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k % Cfg::D), r32);
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
@@ -408,7 +402,10 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& 
                        make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3])));
         }
     } else if (!ragged) {
+        SAT_CLK(o0);
         mbar_wait(&sm.ofree, (ou & 1u) ^ 1u);  // the previous tile's store has read `out`
+        SAT_CLK(o1);
+        if (warp == 0 && lane == 0) WS_ST(kWsFastHits, o1 - o0);
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
             *reinterpret_cast<uint4*>(&sm.out[(row0 + r) * TC + col0]) =
@@ -474,6 +471,9 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg>& sm, const KParams<V>& 
 #pragma unroll
         for (int e = 0; e < E; ++e) acc[e] = V(0);
         bool ddone = ROW ? (I == 0 || J == 0) : true;
+#if SAT_STATS
+        if (p.order & 16) { pend = 0u; ddone = true; }  // timing experiment only: no look-back (wrong sums)
+#endif
         V dacc = V(0);
         int dbase = 1;
         bool cin = false, lpub = false;
@@ -642,6 +642,7 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
             tqf.next();
             --parked;
         }
+        tmem_st_wait();
         tc_fence_before();
         named_bar_sync(2, NW * 32);
         if (warp == 0) tmem_dealloc(sm.tmem_base, Cfg::TM_COLS);
@@ -713,6 +714,7 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 const TileInfo ti = sm.info[tl.s];
                 const bool valid = ti.t < p.ntiles;
                 if (TMA && valid) {
+                    WS_ST(kWsLdIssue, 1);
                     mbar_arrive_expect_tx(&sm.full[sl.s], kTileBytes);
                     tma_load_2d(sm.stage[sl.s], &map_in, &sm.full[sl.s], ti.J * TC, ti.I * TR, policy);
 #if SAT_STATS
@@ -726,7 +728,17 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 progress = true;
                 if (!valid) break;
             }
+#if SAT_STATS
+            if (!progress) {
+                SAT_CLK(b0);
+                __nanosleep(32);
+                SAT_CLK(b1);
+                if (!acq_done && ta.k >= Cfg::NQ) WS_ST(kWsBandBar, b1 - b0);     // ring full: tile slots busy
+                if (tl.k < ta.k) WS_ST(kWsLdEmptyWait, b1 - b0);                 // stage not yet read
+            }
+#else
             if (!progress) __nanosleep(32);
+#endif
         }
     }
 }

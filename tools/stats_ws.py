@@ -25,6 +25,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--n", type=int, default=32768)
 ap.add_argument("--variants", default="0,1")
 ap.add_argument("--dtype", default="f32")
+ap.add_argument("--order", type=int, default=0)
 a = ap.parse_args()
 x = torch.empty((a.n, a.n), dtype=torch.int32, device="cuda")
 satgen.fill_tensor(x, 1447, "f01" if a.dtype == "f32" else "u32")
@@ -32,7 +33,7 @@ if a.dtype == "f32":
     x = x.view(torch.float32)
 y = torch.empty_like(x)
 for v in [int(s) for s in a.variants.split(",")]:
-    sat.set_tuning(v, 0, 0)
+    sat.set_tuning(v, a.order, 0)
     for _ in range(3):
         sat.sat(x, out=y)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
