@@ -170,9 +170,10 @@ int g_ctas_per_sm = 0;
 int g_max_ctas = 0;
 
 int auto_variant(int64_t rows, int64_t cols) {
-    (void)cols;
-    (void)rows;
-    return 0;  // best measured at 32K x 32K (tools/sweep_variants.py)
+    // measured device times (tools/graph_sweep.py, tools/sweep_variants.py): up to
+    // ~1.4K x 1.4K (<= 128 tiles of 128^2) the classic kernel with 64 x 128 tiles has the shortest
+    // latency; above, the TMEM-parked kernel with decoupled walkers (parking depth 4)
+    return rows * cols <= (int64_t(1) << 21) ? 4 : 9;
 }
 
 // ------------------------------------------------------------------ device info caches
