@@ -89,6 +89,26 @@ sat_status_t sat_compute(sat_dtype_t dtype, const void* src, void* dst, int64_t 
 sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,
                               int64_t cols, int64_t pitch, void* stream);
 
+/* ------------------------------------------------------------------ queries on a SAT */
+
+/* Box filter from a SAT b (the O(1) rectangle sum of P:48 that motivates SATs):
+ *   out[i][j] = sum of a[i'][j'] over i' in [i-rh, i+rh] and j' in [j-rw, j+rw], clipped to the
+ *               matrix, = ((b[d][r] - b[u][r]) - b[d][l]) + b[u][l] with u = i-rh-1,
+ *               d = min(i+rh, rows-1), l = j-rw-1, r = min(j+rw, cols-1); entries with a negative
+ *               index are 0.  Evaluated in b's arithmetic (uint32 wraparound / fp32), left to right.
+ *   sat, out  device, rows x cols, row stride `pitch` elements; out must not overlap sat.
+ *   rh, rw    window half-heights / half-widths, >= 0.
+ * Errors: INVALID_VALUE (sizes, negative radius, overlap), MISALIGNED (4-byte), CUDA. */
+sat_status_t sat_box_sum(sat_dtype_t dtype, const void* sat, void* out, int64_t rows, int64_t cols,
+                         int64_t pitch, int64_t rh, int64_t rw, void* stream);
+
+/* Batched rectangle sums: out[k] = sum of a[i][j] for u < i <= d, l < j <= r, where
+ * rects[4k..4k+3] = (u, d, l, r).  Indices are clamped to [-1, rows-1] / [-1, cols-1]; an empty
+ * rectangle gives 0.  rects: device, n x 4 int64, 16-byte aligned; out: device, n elements.
+ * Errors: INVALID_VALUE, MISALIGNED, CUDA. */
+sat_status_t sat_rect_sums(sat_dtype_t dtype, const void* sat, int64_t rows, int64_t cols,
+                           int64_t pitch, const int64_t* rects, int64_t n, void* out, void* stream);
+
 /* ------------------------------------------------------------------ multi-GPU strip partition */
 
 /* Column sums of a strip (not in the paper; BASELINE.json north_star's strip carry):

@@ -15,7 +15,7 @@ Contents (PAPER.md cited as P:<line>; readings R<n> are listed in DESIGN.md):
   the extracted text; reconstructed from their uses at P:144-150, P:162, P:192-243 -- R5),
   each written as the region sum that defines it.
 * ``tile_order`` -- the diagonal-major serial numbering of Fig. 9 (R6).
-* ``rect_sum`` -- the rectangle query of P:48.
+* ``rect_sum`` -- the rectangle query of P:48; ``box_sum`` -- the box filter built from it.
 * ``strip_carry_u32`` / ``strip_carry_f64`` -- the carry row of a horizontal strip (column sums of
   all rows above it), read from the streaming state (R12, multi-GPU).
 * ``f32_tolerance`` -- the fp32 acceptance bound of BASELINE.json north_star (R10).
@@ -202,6 +202,31 @@ def rect_sum(b: np.ndarray, u: int, d: int, l: int, r: int):
     if b.dtype == np.uint32 or b.dtype == np.int32:
         return (at(d, r) - at(u, r) - at(d, l) + at(u, l)) % (1 << 32)
     return at(d, r) - at(u, r) - at(d, l) + at(u, l)
+
+
+def box_sum(b: np.ndarray, rh: int, rw: int) -> np.ndarray:
+    """Box filter from a SAT b: out[i][j] = the P:48 rectangle sum over rows
+    (i-rh-1, min(i+rh, rows-1)] x cols (j-rw-1, min(j+rw, cols-1)], i.e. the input summed over the
+    window [i-rh, i+rh] x [j-rw, j+rw] clipped to the matrix.  Evaluated in b's own arithmetic --
+    uint32 wraparound for integer b, fp32 for float32 b -- left to right as written in P:48:
+    ((b[d][r] - b[u][r]) - b[d][l]) + b[u][l] (reading R17); entries with index -1 are 0."""
+    rows, cols = b.shape
+    if b.dtype == np.float32:
+        bp = np.zeros((rows + 1, cols + 1), dtype=np.float32)
+    else:
+        bp = np.zeros((rows + 1, cols + 1), dtype=np.uint32)
+    bp[1:, 1:] = b if b.dtype == np.float32 else _u32(b)  # bp[x + 1][y + 1] = b[x][y]; index -1 -> 0
+    i = np.arange(rows)
+    j = np.arange(cols)
+    u = np.maximum(i - rh - 1, -1) + 1
+    d = np.minimum(i + rh, rows - 1) + 1
+    l = np.maximum(j - rw - 1, -1) + 1
+    r = np.minimum(j + rw, cols - 1) + 1
+    with np.errstate(over="ignore"):
+        out = bp[d][:, r] - bp[u][:, r]
+        out = out - bp[d][:, l]
+        out = out + bp[u][:, l]
+    return out
 
 
 # ------------------------------------------------------------------------------------ Table II

@@ -21,7 +21,7 @@ from ._lib import SAT_FLOAT32, SAT_INT32, SatError, SatPlan, check
 _lib.lib()  # load now: fail loudly at import if the native library is missing
 
 __all__ = [
-    "sat", "sat_host", "compute", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "sat", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
     "strip_layout", "broadcast_unique_id",
     "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "release_workspaces",
     "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
@@ -102,6 +102,39 @@ def sat_host(src, out=None, *, stream=None):
     check(_lib.lib().sat_compute_host(code, arr.ctypes.data, oarr.ctypes.data, rows, cols, pitch,
                                       _stream_ptr(stream) if torch.cuda.is_available() else None),
           "sat_compute_host")
+    return out
+
+
+def box_sum(b, rh: int, rw: int, out=None, *, stream=None):
+    """Box filter from a SAT ``b``: out[i][j] = sum of the input over the window
+    [i-rh, i+rh] x [j-rw, j+rw] clipped to the matrix.  ``out`` must not be ``b``."""
+    torch = _torch()
+    rows, cols, pitch = _matrix(b, "b")
+    if out is None:
+        out = torch.empty_strided((rows, cols), (pitch, 1), dtype=b.dtype, device=b.device)
+    orows, ocols, opitch = _matrix(out, "out")
+    if (orows, ocols, opitch) != (rows, cols, pitch) or out.dtype != b.dtype or out.device != b.device:
+        raise ValueError("out must match b in shape, row stride, dtype and device")
+    with torch.cuda.device(b.device):
+        check(_lib.lib().sat_box_sum(_dtype_code(b), b.data_ptr(), out.data_ptr(), rows, cols, pitch, rh, rw,
+                                     _stream_ptr(stream)), "sat_box_sum")
+    return out
+
+
+def rect_sums(b, rects, out=None, *, stream=None):
+    """Rectangle sums from a SAT ``b``: ``rects`` is an (n, 4) int64 CUDA tensor of
+    (u, d, l, r), each row giving the sum over u < i <= d, l < j <= r."""
+    torch = _torch()
+    rows, cols, pitch = _matrix(b, "b")
+    if rects.dtype != torch.int64 or rects.dim() != 2 or rects.shape[1] != 4 or not rects.is_contiguous() \
+            or rects.device != b.device:
+        raise ValueError("rects must be a contiguous (n, 4) int64 tensor on b's device")
+    n = rects.shape[0]
+    if out is None:
+        out = torch.empty(n, dtype=b.dtype, device=b.device)
+    with torch.cuda.device(b.device):
+        check(_lib.lib().sat_rect_sums(_dtype_code(b), b.data_ptr(), rows, cols, pitch, rects.data_ptr(), n,
+                                       out.data_ptr(), _stream_ptr(stream)), "sat_rect_sums")
     return out
 
 

@@ -19,6 +19,7 @@
 #include "sat_kernel.cuh"
 #include "sat_ws_kernel.cuh"
 #include "sat_tm_kernel.cuh"
+#include "sat_query_kernels.cuh"
 
 #if defined(SAT_HAVE_NCCL_H)
 #include <nccl.h>
@@ -519,6 +520,66 @@ sat_status_t carry_impl(sat_dtype_t dt, const void* gathered, int nranks, int ra
     return SAT_OK;
 }
 
+// ------------------------------------------------------------------ rectangle queries
+sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, int64_t cols, int64_t pitch, int64_t rh,
+                      int64_t rw, cudaStream_t st) {
+    if (dt != SAT_INT32 && dt != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dt);
+    if (rh < 0 || rw < 0) return fail(SAT_ERR_INVALID_VALUE, "negative box radius");
+    sat_status_t s = validate(b, out, rows, cols, pitch);
+    if (s != SAT_OK || rows == 0 || cols == 0) return s;
+    if (b == out) return fail(SAT_ERR_INVALID_VALUE, "box sums cannot be computed in place");
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    int sms = 0;
+    SAT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int64_t gx = (cols + 1023) / 1024;
+    int64_t gy = (static_cast<int64_t>(sms) * 8 + gx - 1) / gx;
+    if (gy > rows) gy = rows;
+    if (gy > 65535) gy = 65535;
+    const dim3 grid(static_cast<unsigned>(gx), static_cast<unsigned>(gy));
+    const bool vec = ((reinterpret_cast<uintptr_t>(out) & 15u) == 0) && ((pitch * 4) % 16 == 0);
+    if (dt == SAT_INT32) {
+        const uint32_t* bb = static_cast<const uint32_t*>(b);
+        uint32_t* oo = static_cast<uint32_t*>(out);
+        if (vec) sat::box_sum_kernel<uint32_t, true><<<grid, 256, 0, st>>>(bb, oo, rows, cols, pitch, rh, rw);
+        else sat::box_sum_kernel<uint32_t, false><<<grid, 256, 0, st>>>(bb, oo, rows, cols, pitch, rh, rw);
+    } else {
+        const float* bb = static_cast<const float*>(b);
+        float* oo = static_cast<float*>(out);
+        if (vec) sat::box_sum_kernel<float, true><<<grid, 256, 0, st>>>(bb, oo, rows, cols, pitch, rh, rw);
+        else sat::box_sum_kernel<float, false><<<grid, 256, 0, st>>>(bb, oo, rows, cols, pitch, rh, rw);
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "box_sum_kernel");
+    return SAT_OK;
+}
+
+sat_status_t rects_impl(sat_dtype_t dt, const void* b, int64_t rows, int64_t cols, int64_t pitch, const int64_t* rects,
+                        int64_t n, void* out, cudaStream_t st) {
+    if (dt != SAT_INT32 && dt != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dt);
+    if (n < 0 || rows < 0 || cols < 0 || pitch < cols) return fail(SAT_ERR_INVALID_VALUE, "bad sizes");
+    if (n == 0) return SAT_OK;
+    if (!rects || !out || (rows > 0 && cols > 0 && !b)) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    if ((reinterpret_cast<uintptr_t>(rects) & 15u) || (reinterpret_cast<uintptr_t>(out) & 3u) ||
+        (reinterpret_cast<uintptr_t>(b) & 3u))
+        return fail(SAT_ERR_MISALIGNED, "rects must be 16-byte aligned, b and out 4-byte aligned");
+    if (rows == 0 || cols == 0) {
+        SAT_CUDA(cudaMemsetAsync(out, 0, static_cast<size_t>(n) * 4, st));
+        return SAT_OK;
+    }
+    int64_t blocks = (n + 255) / 256;
+    if (blocks > 148 * 32) blocks = 148 * 32;
+    if (dt == SAT_INT32)
+        sat::rect_sums_kernel<uint32_t><<<static_cast<unsigned>(blocks), 256, 0, st>>>(
+            static_cast<const uint32_t*>(b), rows, cols, pitch, rects, n, static_cast<uint32_t*>(out));
+    else
+        sat::rect_sums_kernel<float><<<static_cast<unsigned>(blocks), 256, 0, st>>>(
+            static_cast<const float*>(b), rows, cols, pitch, rects, n, static_cast<float*>(out));
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "rect_sums_kernel");
+    return SAT_OK;
+}
+
 // ------------------------------------------------------------------ end-to-end host pipeline
 struct Staging {
     void* buf = nullptr;
@@ -595,6 +656,16 @@ SAT_API sat_status_t sat_strip_colsum(sat_dtype_t dtype, const void* src, void* 
 SAT_API sat_status_t sat_carry_prefix(sat_dtype_t dtype, const void* gathered, int nranks, int rank, int64_t cols,
                                       void* carry, void* stream) {
     return carry_impl(dtype, gathered, nranks, rank, cols, carry, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_box_sum(sat_dtype_t dtype, const void* sat, void* out, int64_t rows, int64_t cols,
+                                 int64_t pitch, int64_t rh, int64_t rw, void* stream) {
+    return box_impl(dtype, sat, out, rows, cols, pitch, rh, rw, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_rect_sums(sat_dtype_t dtype, const void* sat, int64_t rows, int64_t cols, int64_t pitch,
+                                   const int64_t* rects, int64_t n, void* out, void* stream) {
+    return rects_impl(dtype, sat, rows, cols, pitch, rects, n, out, static_cast<cudaStream_t>(stream));
 }
 
 SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,

@@ -1,0 +1,80 @@
+// sat_query_kernels.cuh -- O(1) rectangle queries on a summed area table.
+//
+// sum_{u < i <= d, l < j <= r} a[i][j] = b[d][r] - b[u][r] - b[d][l] + b[u][l], where b is the SAT
+// of a.  Entries with a row or column index of -1 are zero (the empty prefix).  Evaluated in the
+// SAT's own arithmetic (uint32 wraparound for int32, fp32 for float) left to right:
+// ((b[d][r] - b[u][r]) - b[d][l]) + b[u][l]  (reading R17).
+//
+// box_sum_kernel: the box filter that motivates SATs: out[i][j] = sum of a over the window
+// rows [i-rh, i+rh] x columns [j-rw, j+rw] clipped to the matrix, i.e. P:48 with
+// u = i-rh-1, d = min(i+rh, rows-1), l = j-rw-1, r = min(j+rw, cols-1).  HBM-bound stencil: each SAT
+// row is read by the two output rows that use it (the reuse distance is 2*rh+1 rows, so the second
+// read is an L2 hit for any practical radius); algorithmic bytes 4 read + 4 written per element.
+#pragma once
+
+#include <cstdint>
+
+#include "sat_device.cuh"
+
+namespace sat {
+
+template <typename V>
+__device__ __forceinline__ V sat_at(const V* b, int64_t pitch, int64_t i, int64_t j) {
+    return (i < 0 || j < 0) ? V(0) : __ldg(b + i * pitch + j);
+}
+
+template <typename V>
+__device__ __forceinline__ V rect_from_sat(const V* b, int64_t pitch, int64_t u, int64_t d, int64_t l, int64_t r) {
+    const V drr = sat_at(b, pitch, d, r), urr = sat_at(b, pitch, u, r);
+    const V dll = sat_at(b, pitch, d, l), ull = sat_at(b, pitch, u, l);
+    return ((drr - urr) - dll) + ull;
+}
+
+// One thread: 4 consecutive output columns of one row.  Grid: x over column groups of 4 * blockDim.x,
+// y strides over rows.
+template <typename V, bool VEC>
+__global__ void __launch_bounds__(256) box_sum_kernel(const V* __restrict__ b, V* __restrict__ out, int64_t rows,
+                                                      int64_t cols, int64_t pitch, int64_t rh, int64_t rw) {
+    const int64_t j0 = (static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x) * 4;
+    if (j0 >= cols) return;
+    for (int64_t i = blockIdx.y; i < rows; i += gridDim.y) {
+        const int64_t u = i - rh - 1;
+        const int64_t d = i + rh < rows - 1 ? i + rh : rows - 1;
+        V o[4];
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const int64_t j = j0 + c;
+            const int64_t l = j - rw - 1;
+            const int64_t r = j + rw < cols - 1 ? j + rw : cols - 1;
+            o[c] = (j < cols) ? rect_from_sat(b, pitch, u, d, l, r) : V(0);
+        }
+        V* dst = out + i * pitch + j0;
+        if (VEC && j0 + 3 < cols) {
+            __stcs(reinterpret_cast<uint4*>(dst), make_uint4(to_bits(o[0]), to_bits(o[1]), to_bits(o[2]), to_bits(o[3])));
+        } else {
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                if (j0 + c < cols) dst[c] = o[c];
+        }
+    }
+}
+
+// Batched rectangle queries: rects[k] = (u, d, l, r) in the convention of P:48 (u < i <= d,
+// l < j <= r).  Indices are clamped into [-1, rows-1] / [-1, cols-1] (memory safety); an empty
+// rectangle (u >= d or l >= r after clamping) gives 0.
+template <typename V>
+__global__ void __launch_bounds__(256) rect_sums_kernel(const V* __restrict__ b, int64_t rows, int64_t cols,
+                                                        int64_t pitch, const int64_t* __restrict__ rects, int64_t n,
+                                                        V* __restrict__ out) {
+    for (int64_t k = static_cast<int64_t>(blockIdx.x) * blockDim.x + threadIdx.x; k < n;
+         k += static_cast<int64_t>(gridDim.x) * blockDim.x) {
+        const longlong2 ud = *reinterpret_cast<const longlong2*>(rects + 4 * k);
+        const longlong2 lr = *reinterpret_cast<const longlong2*>(rects + 4 * k + 2);
+        auto clampi = [](int64_t x, int64_t hi) { return x < -1 ? int64_t(-1) : (x > hi ? hi : x); };
+        const int64_t u = clampi(ud.x, rows - 1), d = clampi(ud.y, rows - 1);
+        const int64_t l = clampi(lr.x, cols - 1), r = clampi(lr.y, cols - 1);
+        out[k] = (u >= d || l >= r) ? V(0) : rect_from_sat(b, pitch, u, d, l, r);
+    }
+}
+
+}  // namespace sat

@@ -443,3 +443,77 @@ def test_sharded_nccl_single_rank():
     status, err = q.get(timeout=240)
     proc.join(timeout=60)
     assert status == "ok", err
+
+
+# ----------------------------------------------------------------------------- queries on a SAT
+@pytest.mark.parametrize("shape,pitch,rh,rw", [((1, 1), None, 0, 0), ((300, 517), None, 3, 5), ((129, 257), 264, 0, 7),
+                                               ((64, 1000), None, 40, 1), ((1009, 203), 208, 12, 12),
+                                               ((50, 60), None, 100, 100)])
+def test_box_sum_int32_bit_exact(sat, shape, pitch, rh, rw):
+    b = satgen.gen_host(*shape, seed=31 + shape[0], dist="u32")  # any matrix is a valid operand of P:48
+    buf, bd = dev_copy(b, pitch)
+    obuf, od = dev_copy(np.zeros_like(b), pitch)
+    sat.box_sum(bd, rh, rw, out=od)
+    torch.cuda.synchronize()
+    got = od.cpu().numpy().view(np.uint32)
+    want = oracle.box_sum(b.view(np.uint32), rh, rw)
+    assert (got == want).all()
+    if pitch is not None and pitch > shape[1]:
+        full = obuf[: shape[0] * pitch].view(shape[0], pitch)
+        assert (full[:, shape[1]:] == 0x5A5A5A5A).all(), "pad elements were written"
+
+
+@pytest.mark.parametrize("shape,rh,rw", [((333, 444), 4, 9), ((128, 128), 0, 0), ((1, 2049), 0, 30)])
+def test_box_sum_fp32_bit_exact(sat, shape, rh, rw):
+    b = satgen.gen_host(*shape, seed=77, dist="fsym")
+    _, bd = dev_copy(b)
+    got = sat.box_sum(bd, rh, rw).cpu().numpy()
+    want = oracle.box_sum(b, rh, rw)  # same fp32 operations in the same order
+    assert (got.view(np.uint32) == want.view(np.uint32)).all()
+
+
+def test_box_filter_end_to_end_from_gpu_sat(sat):
+    a = satgen.gen_host(700, 900, seed=5, dist="u32")
+    b = sat.sat(torch.from_numpy(a).cuda())
+    got = sat.box_sum(b, 6, 11).cpu().numpy().view(np.uint32)
+    want = oracle.box_sum(oracle.sat_u32(a), 6, 11)  # oracle SAT, oracle box formula
+    assert (got == want).all()
+    # spot entries against the direct window sum (the definition)
+    for i, j in [(0, 0), (699, 899), (350, 5), (3, 450)]:
+        assert int(got[i, j]) == int(a.view(np.uint32)[max(0, i - 6): i + 7, max(0, j - 11): j + 12].astype(np.uint64).sum()) % (1 << 32)
+
+
+def test_rect_sums_int32_and_fp32(sat):
+    rng = np.random.default_rng(9)
+    for dist in ("u32", "fsym"):
+        b = satgen.gen_host(257, 301, seed=123, dist=dist)
+        _, bd = dev_copy(b)
+        rows, cols = b.shape
+        n = 5000
+        r = np.stack([rng.integers(-3, rows + 3, n), rng.integers(-3, rows + 3, n),
+                      rng.integers(-3, cols + 3, n), rng.integers(-3, cols + 3, n)], axis=1).astype(np.int64)
+        r[:100, 1] = r[:100, 0]  # empty rectangles
+        got = sat.rect_sums(bd, torch.from_numpy(r).cuda()).cpu().numpy()
+        for k in range(n):
+            u = min(max(r[k, 0], -1), rows - 1); d = min(max(r[k, 1], -1), rows - 1)
+            l = min(max(r[k, 2], -1), cols - 1); rr = min(max(r[k, 3], -1), cols - 1)
+            if u >= d or l >= rr:
+                want = 0
+            elif dist == "u32":
+                want = oracle.rect_sum(b.view(np.uint32), u, d, l, rr)
+            else:
+                z = np.float32(0)
+                at = lambda x, y: z if (x < 0 or y < 0) else b[x, y]  # noqa: E731
+                want = ((at(d, rr) - at(u, rr)) - at(d, l)) + at(u, l)
+            if dist == "u32":
+                assert int(got.view(np.uint32)[k]) == int(want), k
+            else:
+                assert got[k] == np.float32(want), k
+
+
+def test_query_errors(sat):
+    x = torch.zeros((8, 8), dtype=torch.int32, device="cuda")
+    with pytest.raises(sat.SatError):
+        sat.box_sum(x, -1, 0)
+    with pytest.raises(sat.SatError):
+        sat.box_sum(x, 1, 1, out=x)

@@ -107,6 +107,41 @@ def test_rectangle_formula_all_rectangles():
             assert oracle.region_sum(a, u + 1, d, l + 1, r) == want
 
 
+
+def brute_box(a: np.ndarray, rh: int, rw: int) -> np.ndarray:
+    """Window sums by direct summation of the clipped window (exact Python ints)."""
+    rows, cols = a.shape
+    ai = a.astype(np.int64)
+    out = np.zeros((rows, cols), dtype=object)
+    for i in range(rows):
+        for j in range(cols):
+            out[i, j] = int(ai[max(0, i - rh): i + rh + 1, max(0, j - rw): j + rw + 1].sum())
+    return out
+
+
+@pytest.mark.parametrize("shape,rh,rw", [((1, 1), 0, 0), ((7, 9), 1, 2), ((12, 5), 3, 0), ((6, 6), 10, 10),
+                                         ((9, 13), 0, 4), ((16, 11), 2, 7)])
+def test_box_sum_is_the_clipped_window_sum(shape, rh, rw):
+    a = RNG.integers(0, MOD, size=shape, dtype=np.uint64).astype(np.uint32)
+    got = oracle.box_sum(oracle.sat_u32(a), rh, rw)
+    want = np.vectorize(lambda x: x % MOD)(brute_box(a, rh, rw)).astype(np.uint64)
+    assert (got.astype(np.uint64) == want).all()
+
+
+def test_box_sum_fp32_exact_regime_and_association():
+    # small integers in fp32: every SAT entry and every partial of the P:48 formula is exact
+    a = RNG.integers(0, 4, size=(23, 31)).astype(np.float32)
+    b = oracle.sat_f64(a).astype(np.float32)
+    got = oracle.box_sum(b, 2, 3)
+    assert got.dtype == np.float32
+    assert (got.astype(np.float64) == brute_box(a, 2, 3).astype(np.float64)).all()
+    # evaluation order is ((drr - urr) - dll) + ull in fp32: check one entry against that by hand
+    b = RNG.standard_normal((5, 6)).astype(np.float32) * np.float32(1e4)
+    o = oracle.box_sum(b, 1, 1)
+    i, j = 3, 4  # u = 1, d = 4, l = 2, r = 5
+    want = ((b[4, 5] - b[1, 5]) - b[4, 2]) + b[1, 2]
+    assert o[i, j] == want
+
 # ----------------------------------------------------------------------------- closed forms
 def test_all_ones():
     a = np.ones((37, 53), dtype=np.int32)
