@@ -72,6 +72,17 @@ sat_status_t sat_compute_i32(const int32_t* src, int32_t* dst, int64_t rows, int
 sat_status_t sat_compute_f32(const float* src, float* dst, int64_t rows, int64_t cols,
                              int64_t pitch, void* stream);
 
+/* Integral image of an 8-bit image (the computer-vision use of SATs): src is u8, the SAT
+ * is uint32 (exact while the total stays below 2^32, i.e. rows*cols*255 < 2^32; modulo 2^32
+ * beyond, like sat_compute_i32).  Same single-pass method; 1 B read + 4 B written per element.
+ *   src        device, rows x cols bytes, row stride src_pitch BYTES (>= cols).
+ *   dst        device, rows x cols uint32, row stride `pitch` ELEMENTS (>= cols); must not overlap src.
+ * 16-byte aligned src/dst with src_pitch % 16 == 0 and pitch*4 % 16 == 0 take the TMA path, any other
+ * layout the generic path.  Errors: INVALID_VALUE (sizes, overlap), MISALIGNED (dst not 4-byte
+ * aligned), UNSUPPORTED (a forced variant without u8 support), OUT_OF_MEMORY, CUDA. */
+sat_status_t sat_compute_u8(const uint8_t* src, int64_t src_pitch, uint32_t* dst, int64_t rows,
+                            int64_t cols, int64_t pitch, void* stream);
+
 /* Same as above for either dtype, plus an optional carry row.
  *   carry  device, `cols` elements of the same dtype, or NULL.  When given, carry[j] is added to
  *          every element of column j of the result: dst[i][j] = carry[j] + SAT(src)[i][j].  With

@@ -21,7 +21,7 @@ from ._lib import SAT_FLOAT32, SAT_INT32, SatError, SatPlan, check
 _lib.lib()  # load now: fail loudly at import if the native library is missing
 
 __all__ = [
-    "sat", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "sat", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
     "strip_layout", "broadcast_unique_id",
     "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "release_workspaces",
     "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
@@ -102,6 +102,26 @@ def sat_host(src, out=None, *, stream=None):
     check(_lib.lib().sat_compute_host(code, arr.ctypes.data, oarr.ctypes.data, rows, cols, pitch,
                                       _stream_ptr(stream) if torch.cuda.is_available() else None),
           "sat_compute_host")
+    return out
+
+
+def sat_u8(src, out=None, *, stream=None):
+    """Integral image of a 2-D uint8 CUDA tensor: uint32 SAT returned as an int32 tensor holding the
+    uint32 bit patterns (exact while the total is < 2^32, modulo 2^32 beyond)."""
+    torch = _torch()
+    if src.dtype != torch.uint8:
+        raise TypeError("sat_u8 needs a uint8 tensor")
+    rows, cols, spitch = _matrix(src, "src")
+    if out is None:
+        out = torch.empty((rows, cols), dtype=torch.int32, device=src.device)
+    if out.dtype != torch.int32 or out.device != src.device:
+        raise ValueError("out must be an int32 tensor on src's device")
+    orows, ocols, opitch = _matrix(out, "out")
+    if (orows, ocols) != (rows, cols):
+        raise ValueError("out must have src's shape")
+    with torch.cuda.device(src.device):
+        check(_lib.lib().sat_compute_u8(src.data_ptr(), spitch, out.data_ptr(), rows, cols, opitch,
+                                        _stream_ptr(stream)), "sat_compute_u8")
     return out
 
 

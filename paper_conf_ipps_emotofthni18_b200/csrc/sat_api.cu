@@ -9,6 +9,7 @@
 #include <map>
 #include <mutex>
 #include <string>
+#include <type_traits>
 #include <utility>
 #include <vector>
 
@@ -64,8 +65,8 @@ struct Variant {
     int TR, TC, NW, STAGES;
     int family;            // 2 = TMEM-parked (sat_tm_kernel), 1 = warp-specialised (sat_ws_kernel), 0 = classic
     size_t smem;           // dynamic shared memory bytes (same for int32 / fp32)
-    LaunchFn launch[2];    // [dtype]
-    PrepareFn prepare[2];  // [dtype]
+    LaunchFn launch[3];    // [dtype]; [kU8] = u8 input -> uint32 SAT (TMEM-parked family only, else null)
+    PrepareFn prepare[3];  // [dtype]
 };
 
 // Kernel family traits: the classic kernel (sat_kernel.cuh, TileCfg) and the warp-specialised
@@ -104,7 +105,16 @@ struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT>> {
     static constexpr size_t smem() { return sizeof(sat::TmSmem<V, Cfg>); }
     template <typename V, bool TMA, bool CARRY>
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_tm_kernel<V, Cfg, TMA, CARRY>); }
+    // u8 pixels in, uint32 integral image out
+    static constexpr size_t smem_u8() { return sizeof(sat::TmSmem<uint32_t, Cfg, uint8_t>); }
+    template <bool TMA, bool CARRY>
+    static void* kernel_u8() { return reinterpret_cast<void*>(&sat::sat_tm_kernel<uint32_t, Cfg, TMA, CARRY, uint8_t>); }
 };
+
+template <typename F, typename = void>
+struct HasU8 { static constexpr bool value = false; };
+template <typename F>
+struct HasU8<F, std::void_t<decltype(F::smem_u8())>> { static constexpr bool value = true; };
 
 template <typename V, typename F>
 void* pick_kernel(bool tma, bool carry) {
@@ -131,6 +141,33 @@ cudaError_t prepare_variant(bool tma, bool carry, int* occupancy) {
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy, k, F::threads, smem);
 }
 
+constexpr int kU8 = 2;  // internal dtype index: u8 input, uint32 output
+
+template <typename F>
+void* pick_kernel_u8(bool tma, bool carry) {
+    return tma ? (carry ? F::template kernel_u8<true, true>() : F::template kernel_u8<true, false>())
+               : (carry ? F::template kernel_u8<false, true>() : F::template kernel_u8<false, false>());
+}
+
+template <typename Cfg>
+cudaError_t launch_variant_u8(bool tma, bool carry, dim3 grid, cudaStream_t st, const CUtensorMap& mi,
+                              const CUtensorMap& mo, const void* params) {
+    using F = Family<Cfg>;
+    const KParams<uint32_t>& p = *static_cast<const KParams<uint32_t>*>(params);
+    void* args[] = {const_cast<CUtensorMap*>(&mi), const_cast<CUtensorMap*>(&mo), const_cast<KParams<uint32_t>*>(&p)};
+    return cudaLaunchKernel(pick_kernel_u8<F>(tma, carry), grid, dim3(F::threads), args, F::smem_u8(), st);
+}
+
+template <typename Cfg>
+cudaError_t prepare_variant_u8(bool tma, bool carry, int* occupancy) {
+    using F = Family<Cfg>;
+    void* k = pick_kernel_u8<F>(tma, carry);
+    const int smem = static_cast<int>(F::smem_u8());
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy, k, F::threads, smem);
+}
+
 template <typename Cfg>
 Variant make_variant() {
     Variant v;
@@ -144,6 +181,13 @@ Variant make_variant() {
     v.launch[SAT_FLOAT32] = &launch_variant<float, Cfg>;
     v.prepare[SAT_INT32] = &prepare_variant<uint32_t, Cfg>;
     v.prepare[SAT_FLOAT32] = &prepare_variant<float, Cfg>;
+    if constexpr (HasU8<Family<Cfg>>::value) {
+        v.launch[kU8] = &launch_variant_u8<Cfg>;
+        v.prepare[kU8] = &prepare_variant_u8<Cfg>;
+    } else {
+        v.launch[kU8] = nullptr;
+        v.prepare[kU8] = nullptr;
+    }
     return v;
 }
 
@@ -159,6 +203,7 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<16, 3, 8, 1, 3, 4, 1>>(),  // 7
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 8
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),  // 9
+        make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>>(),  // 10: u8 integral images only (4 stages of 16 KiB u8 tiles)
     };
     return vs;
 }
@@ -195,7 +240,7 @@ sat_status_t device_info(int dev, DeviceInfo** out) {
     return SAT_OK;
 }
 
-sat_status_t occupancy(int dev, int vi, sat_dtype_t dt, bool tma, bool carry, int* occ) {
+sat_status_t occupancy(int dev, int vi, int dt, bool tma, bool carry, int* occ) {
     DeviceInfo* di;
     sat_status_t s = device_info(dev, &di);
     if (s != SAT_OK) return s;
@@ -203,7 +248,12 @@ sat_status_t occupancy(int dev, int vi, sat_dtype_t dt, bool tma, bool carry, in
     auto it = di->occ.find(key);
     if (it == di->occ.end()) {
         int o = 0;
+        if (!variants()[vi].prepare[dt]) return fail(SAT_ERR_UNSUPPORTED, "kernel variant %d lacks this dtype", vi);
         cudaError_t e = variants()[vi].prepare[dt](tma, carry, &o);
+        if (e == cudaErrorInvalidValue) {  // dynamic shared memory above the per-block limit
+            cudaGetLastError();
+            return fail(SAT_ERR_UNSUPPORTED, "kernel variant %d does not fit on an SM for this dtype", vi);
+        }
         if (e != cudaSuccess) return cuda_fail(e, "kernel attribute / occupancy query");
         if (o < 1) return fail(SAT_ERR_UNSUPPORTED, "kernel variant %d does not fit on an SM", vi);
         it = di->occ.emplace(key, o).first;
@@ -331,6 +381,19 @@ sat_status_t encode_map(CUtensorMap* m, sat_dtype_t dt, const void* ptr, int64_t
     return SAT_OK;
 }
 
+sat_status_t encode_map_u8(CUtensorMap* m, const void* ptr, int64_t rows, int64_t cols, int64_t pitch_bytes, int TR,
+                           int TC) {
+    cuuint64_t dims[2] = {static_cast<cuuint64_t>(cols), static_cast<cuuint64_t>(rows)};
+    cuuint64_t strides[1] = {static_cast<cuuint64_t>(pitch_bytes)};
+    cuuint32_t box[2] = {static_cast<cuuint32_t>(TC), static_cast<cuuint32_t>(TR)};
+    cuuint32_t estr[2] = {1u, 1u};
+    CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<void*>(ptr), dims, strides, box, estr,
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return fail(SAT_ERR_CUDA, "cuTensorMapEncodeTiled (u8) failed (CUresult %d)", (int)r);
+    return SAT_OK;
+}
+
 // ------------------------------------------------------------------ validation / planning
 sat_status_t validate(const void* src, const void* dst, int64_t rows, int64_t cols, int64_t pitch) {
     if (rows < 0 || cols < 0 || pitch < cols)
@@ -361,11 +424,12 @@ struct Plan {
     bool tma;
 };
 
-sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* src, const void* dst, Plan* pl) {
+sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* src, const void* dst, Plan* pl,
+                       bool u8 = false, int64_t src_pitch = 0) {
     int vi, order;
     {
         std::lock_guard<std::mutex> lk(g_mu);
-        vi = g_variant >= 0 ? g_variant : auto_variant(rows, cols);
+        vi = g_variant >= 0 ? g_variant : (u8 ? 10 : auto_variant(rows, cols));
         order = g_order;
     }
     const Variant& v = variants()[vi];
@@ -376,21 +440,43 @@ sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* sr
     pl->C = static_cast<int>((cols + v.TC - 1) / v.TC);
     pl->ntiles = static_cast<int64_t>(pl->R) * pl->C;
     pl->order = order;
-    pl->tma = tma_ok(src, dst, pitch);
+    pl->tma = u8 ? (((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15u) == 0 &&
+                    src_pitch % 16 == 0 && (pitch * 4) % 16 == 0 && pitch * 4 < (int64_t(1) << 40) &&
+                    src_pitch < (int64_t(1) << 40))
+                 : tma_ok(src, dst, pitch);
     if (pl->ntiles > (int64_t(1) << 31) - 4096)
         return fail(SAT_ERR_UNSUPPORTED, "too many tiles (%lld)", (long long)pl->ntiles);
     return SAT_OK;
 }
 
 // ------------------------------------------------------------------ the hot path
-sat_status_t compute_impl(sat_dtype_t dt, const void* src, void* dst, int64_t rows, int64_t cols, int64_t pitch,
-                          const void* carry, cudaStream_t st) {
-    if (dt != SAT_INT32 && dt != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dt);
-    sat_status_t s = validate(src, dst, rows, cols, pitch);
+sat_status_t validate_u8(const void* src, int64_t src_pitch, const void* dst, int64_t rows, int64_t cols,
+                         int64_t pitch) {
+    if (rows < 0 || cols < 0 || pitch < cols || src_pitch < cols)
+        return fail(SAT_ERR_INVALID_VALUE, "bad sizes rows=%lld cols=%lld pitch=%lld src_pitch=%lld", (long long)rows,
+                    (long long)cols, (long long)pitch, (long long)src_pitch);
+    if (rows == 0 || cols == 0) return SAT_OK;
+    if (!src || !dst) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    if (reinterpret_cast<uintptr_t>(dst) & 3u) return fail(SAT_ERR_MISALIGNED, "dst must be 4-byte aligned");
+    const uintptr_t a = reinterpret_cast<uintptr_t>(src), b = reinterpret_cast<uintptr_t>(dst);
+    const uintptr_t na = static_cast<uintptr_t>((rows - 1) * src_pitch + cols);
+    const uintptr_t nb = static_cast<uintptr_t>(((rows - 1) * pitch + cols) * 4);
+    if (a < b + nb && b < a + na) return fail(SAT_ERR_INVALID_VALUE, "src and dst overlap");
+    if (rows > (int64_t(1) << 31) - 1 || cols > (int64_t(1) << 31) - 1)
+        return fail(SAT_ERR_UNSUPPORTED, "rows and cols must be < 2^31");
+    return SAT_OK;
+}
+
+// dt: SAT_INT32, SAT_FLOAT32, or kU8 (u8 input with row stride src_pitch bytes -> uint32 output)
+sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int64_t cols, int64_t pitch,
+                          const void* carry, cudaStream_t st, int64_t src_pitch = 0) {
+    if (dt != SAT_INT32 && dt != SAT_FLOAT32 && dt != kU8) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", dt);
+    const bool u8 = dt == kU8;
+    sat_status_t s = u8 ? validate_u8(src, src_pitch, dst, rows, cols, pitch) : validate(src, dst, rows, cols, pitch);
     if (s != SAT_OK || rows == 0 || cols == 0) return s;
     if (carry && (reinterpret_cast<uintptr_t>(carry) & 3u)) return fail(SAT_ERR_MISALIGNED, "carry misaligned");
     Plan pl;
-    if ((s = make_plan(rows, cols, pitch, src, dst, &pl)) != SAT_OK) return s;
+    if ((s = make_plan(rows, cols, pitch, src, dst, &pl, u8, src_pitch)) != SAT_OK) return s;
     const Variant& v = variants()[pl.vi];
 
     int dev = 0;
@@ -414,8 +500,15 @@ sat_status_t compute_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ro
     std::memset(&mo, 0, sizeof(mo));
     if (pl.tma) {
         if ((s = get_encoder()) != SAT_OK) return s;
-        if ((s = encode_map(&mi, dt, src, rows, cols, pitch, v.TR, v.TC)) != SAT_OK) return s;
-        if ((s = encode_map(&mo, dt, dst, rows, cols, pitch, v.TR, v.TC)) != SAT_OK) return s;
+        if (u8) {
+            if ((s = encode_map_u8(&mi, src, rows, cols, src_pitch, v.TR, v.TC)) != SAT_OK) return s;
+            if ((s = encode_map(&mo, SAT_INT32, dst, rows, cols, pitch, v.TR, v.TC)) != SAT_OK) return s;
+        } else {
+            if ((s = encode_map(&mi, static_cast<sat_dtype_t>(dt), src, rows, cols, pitch, v.TR, v.TC)) != SAT_OK)
+                return s;
+            if ((s = encode_map(&mo, static_cast<sat_dtype_t>(dt), dst, rows, cols, pitch, v.TR, v.TC)) != SAT_OK)
+                return s;
+        }
     }
     KParams<uint32_t> p;  // identical layout for float
     p.src = static_cast<const uint32_t*>(src);
@@ -434,6 +527,9 @@ sat_status_t compute_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ro
     p.carry = static_cast<const uint32_t*>(carry);
     p.stats = nullptr;
     p.trace = nullptr;
+    p.src8 = u8 ? static_cast<const uint8_t*>(src) : nullptr;
+    p.src_pitch = u8 ? src_pitch : pitch;
+    if (u8) p.src = nullptr;
 #if SAT_STATS
     {
         const size_t need = static_cast<size_t>(grid) * sat::kNumStats + 8 * static_cast<size_t>(pl.ntiles);
@@ -646,6 +742,11 @@ SAT_API sat_status_t sat_compute_i32(const int32_t* src, int32_t* dst, int64_t r
 SAT_API sat_status_t sat_compute_f32(const float* src, float* dst, int64_t rows, int64_t cols, int64_t pitch,
                                      void* stream) {
     return compute_impl(SAT_FLOAT32, src, dst, rows, cols, pitch, nullptr, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_compute_u8(const uint8_t* src, int64_t src_pitch, uint32_t* dst, int64_t rows, int64_t cols,
+                                    int64_t pitch, void* stream) {
+    return compute_impl(kU8, src, dst, rows, cols, pitch, nullptr, static_cast<cudaStream_t>(stream), src_pitch);
 }
 
 SAT_API sat_status_t sat_strip_colsum(sat_dtype_t dtype, const void* src, void* colsum, int64_t rows, int64_t cols,

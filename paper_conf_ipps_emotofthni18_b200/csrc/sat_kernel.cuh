@@ -74,6 +74,8 @@ struct KParams {
     const V* carry;    // [cols] or nullptr
     long long* stats;  // [gridDim.x][kNumStats] (SAT_STATS builds only) or nullptr
     long long* trace;  // [ntiles][2]: acquisition / store-issue globaltimer ns (SAT_STATS builds only)
+    const uint8_t* src8;  // u8 input (integral images, sat_compute_u8): generic path only, else nullptr
+    int64_t src_pitch;    // row stride of src8 in bytes
 };
 
 __device__ __forceinline__ uint64_t pack(uint32_t epoch, uint32_t kind, uint32_t bits) {

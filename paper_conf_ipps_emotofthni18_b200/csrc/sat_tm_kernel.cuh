@@ -52,9 +52,9 @@ struct TmCfg {
     static_assert(IN >= 1 && NQ >= IN + D - 1 && NQ <= 16, "rings");
 };
 
-template <typename V, typename Cfg>
+template <typename V, typename Cfg, typename TIn = V>
 struct TmSmem {
-    alignas(1024) V stage[Cfg::IN][Cfg::TR * Cfg::TC];  // input ring (TMA loads)
+    alignas(1024) TIn stage[Cfg::IN][Cfg::TR * Cfg::TC];  // input ring (TMA loads; u8 for integral images)
     alignas(1024) V out[Cfg::DIRECT ? 4 : Cfg::TR * Cfg::TC];  // GSAT of one tile (TMA store source)
     alignas(16) V band[2][Cfg::NW][Cfg::TC];
     alignas(16) V rp[Cfg::NQ][Cfg::TR];
@@ -156,8 +156,8 @@ __device__ __forceinline__ uint32_t tm_addr(uint32_t base, int warp, int slot) {
 
 // Step 1 + local SAT + Steps 2.A.1 / 2.B.1 of tile k (input stage sl, tile slot tq); parks the block in
 // TMEM slot k % D.  Returns false at the end marker.
-template <typename V, typename Cfg, bool TMA>
-__device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p, const Slot<Cfg::IN>& sl,
+template <typename V, typename Cfg, bool TMA, typename TIn>
+__device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, const Slot<Cfg::IN>& sl,
                                          const Slot<Cfg::NQ>& tq, uint32_t epoch, int warp, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
     const int s = sl.s;
@@ -175,8 +175,17 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p
     const long long tidx = static_cast<long long>(I) * p.C + J;
     const int par = tq.k & 1;
     V v[RPW][4];
-    if constexpr (TMA) {
-        const V* tile = sm.stage[s];
+    if constexpr (TMA && sizeof(TIn) == 1) {
+        // u8 pixels (integral image): a lane's 4 columns are one 32-bit word of the stage row
+        const TIn* tile = sm.stage[s];
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const uint32_t w = *reinterpret_cast<const uint32_t*>(&tile[(row0 + r) * TC + col0]);
+#pragma unroll
+            for (int c = 0; c < 4; ++c) v[r][c] = V((w >> (8 * c)) & 0xffu);
+        }
+    } else if constexpr (TMA) {
+        const TIn* tile = sm.stage[s];
 #pragma unroll
         for (int r = 0; r < RPW; ++r) {
             const uint4 q = *reinterpret_cast<const uint4*>(&tile[(row0 + r) * TC + col0]);
@@ -190,7 +199,9 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p
 #pragma unroll
             for (int c = 0; c < 4; ++c) {
                 const long long gj = static_cast<long long>(J) * TC + col0 + c;
-                v[r][c] = (gi < p.rows && gj < p.cols) ? p.src[gi * p.pitch + gj] : V(0);
+                const bool in = gi < p.rows && gj < p.cols;
+                if constexpr (sizeof(TIn) == 1) v[r][c] = in ? V(p.src8[gi * p.src_pitch + gj]) : V(0);
+                else v[r][c] = in ? p.src[gi * p.pitch + gj] : V(0);
             }
         }
     }
@@ -316,8 +327,8 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg>& sm, const KParams<V>& p
 
 // Steps 2.A.3 / 2.B.3 / 3.1 / 3.3 and Step 4 of tile k (tile slot tq; its block parked in TMEM slot
 // k % D), GSAT into the output buffer (use number `ou` of it).
-template <typename V, typename Cfg, bool TMA, bool CARRY>
-__device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& p, const Slot<Cfg::NQ>& tq,
+template <typename V, typename Cfg, bool TMA, bool CARRY, typename TIn>
+__device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, const Slot<Cfg::NQ>& tq,
                                           uint32_t ou, uint32_t epoch, int warp, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
     const int q = tq.s;
@@ -450,8 +461,8 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg>& sm, const KParams<V>& 
 // walk is empty, only ever publish GS).  A diagonal look-back therefore sums GLS words up to
 // the first GS word (reading R8) instead of waiting for GS(I-1,J-1): no chain in any of the
 // three directions waits for a neighbour's completion.
-template <typename V, typename Cfg, bool ROW>
-__device__ __forceinline__ void tm_walker(TmSmem<V, Cfg>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
+template <typename V, typename Cfg, bool ROW, typename TIn>
+__device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, RPW = Cfg::RPW, NW = Cfg::NW;
     constexpr int E = ROW ? Cfg::ER : Cfg::EC;
     constexpr int DW = 4;  // diagonal predecessors polled per round
@@ -574,14 +585,14 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg>& sm, const KParams<V>& 
     }
 }
 
-template <typename V, typename Cfg, bool TMA, bool CARRY>
+template <typename V, typename Cfg, bool TMA, bool CARRY, typename TIn = V>
 __global__ void __launch_bounds__(Cfg::THREADS, 1)
 sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant__ CUtensorMap map_out,
               const KParams<V> p) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, IN = Cfg::IN;
-    constexpr uint32_t kTileBytes = TR * TC * sizeof(V);
+    constexpr uint32_t kTileBytes = TR * TC * sizeof(TIn);
     extern __shared__ __align__(1024) unsigned char smem_raw[];
-    TmSmem<V, Cfg>& sm = *reinterpret_cast<TmSmem<V, Cfg>*>(smem_raw);
+    TmSmem<V, Cfg, TIn>& sm = *reinterpret_cast<TmSmem<V, Cfg, TIn>*>(smem_raw);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
 #if SAT_STATS
@@ -627,17 +638,17 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         int parked = 0;
         bool more = true;
         while (more && parked < Cfg::D - 1) {
-            more = tm_local<V, Cfg, TMA>(sm, p, sl, tql, epoch, warp, lane);
+            more = tm_local<V, Cfg, TMA, TIn>(sm, p, sl, tql, epoch, warp, lane);
             if (more) { ++parked; sl.next(); tql.next(); }
         }
         while (parked > 0) {
             if (more) {
-                more = tm_local<V, Cfg, TMA>(sm, p, sl, tql, epoch, warp, lane);
+                more = tm_local<V, Cfg, TMA, TIn>(sm, p, sl, tql, epoch, warp, lane);
                 if (more) { ++parked; sl.next(); tql.next(); }
             }
             const TileInfo ti = sm.info[tqf.s];
             const bool ragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
-            tm_finish<V, Cfg, TMA, CARRY>(sm, p, tqf, ou, epoch, warp, lane);
+            tm_finish<V, Cfg, TMA, CARRY, TIn>(sm, p, tqf, ou, epoch, warp, lane);
             if (!ragged) ++ou;
             tqf.next();
             --parked;
@@ -647,10 +658,10 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         named_bar_sync(2, NW * 32);
         if (warp == 0) tmem_dealloc(sm.tmem_base, Cfg::TM_COLS);
     } else if (warp == Cfg::ROW_WARP) {
-        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, true>(sm, p, epoch, lane);
+        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, true, TIn>(sm, p, epoch, lane);
         else ws_walker<V, Cfg, true>(sm, p, epoch, lane);
     } else if (warp == Cfg::COL_WARP) {
-        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, false>(sm, p, epoch, lane);
+        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, false, TIn>(sm, p, epoch, lane);
         else ws_walker<V, Cfg, false>(sm, p, epoch, lane);
     } else if (warp == Cfg::STORE_WARP) {
         // ================================================================ storer (one lane)
