@@ -63,6 +63,7 @@ using PrepareFn = cudaError_t (*)(bool tma, bool carry, int* occupancy);
 
 struct Variant {
     int TR, TC, NW, STAGES;
+    int OBR;               // rows of the output TMA box (TR, or TR/4 for quarter stores)
     int family;            // 2 = TMEM-parked (sat_tm_kernel), 1 = warp-specialised (sat_ws_kernel), 0 = classic
     size_t smem;           // dynamic shared memory bytes (same for int32 / fp32)
     LaunchFn launch[3];    // [dtype]; [kU8] = u8 input -> uint32 SAT (TMEM-parked family only, else null)
@@ -96,9 +97,10 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
 };
 
-template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT>
-struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT>> {
-    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT>;
+template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS>;
+    static constexpr int out_box_rows = Cfg::OBR;
     static constexpr int threads = Cfg::THREADS;
     static constexpr int family = 2;
     template <typename V>
@@ -110,6 +112,11 @@ struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT>> {
     template <bool TMA, bool CARRY>
     static void* kernel_u8() { return reinterpret_cast<void*>(&sat::sat_tm_kernel<uint32_t, Cfg, TMA, CARRY, uint8_t>); }
 };
+
+template <typename F, typename = void>
+struct HasOBR { static constexpr bool value = false; };
+template <typename F>
+struct HasOBR<F, std::void_t<decltype(F::out_box_rows)>> { static constexpr bool value = true; };
 
 template <typename F, typename = void>
 struct HasU8 { static constexpr bool value = false; };
@@ -176,6 +183,8 @@ Variant make_variant() {
     v.NW = Cfg::NW;
     v.STAGES = Cfg::STAGES;
     v.family = Family<Cfg>::family;
+    if constexpr (HasOBR<Family<Cfg>>::value) v.OBR = Family<Cfg>::out_box_rows;
+    else v.OBR = Cfg::TR;
     v.smem = Family<Cfg>::template smem<uint32_t>();
     v.launch[SAT_INT32] = &launch_variant<uint32_t, Cfg>;
     v.launch[SAT_FLOAT32] = &launch_variant<float, Cfg>;
@@ -502,11 +511,11 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
         if ((s = get_encoder()) != SAT_OK) return s;
         if (u8) {
             if ((s = encode_map_u8(&mi, src, rows, cols, src_pitch, v.TR, v.TC)) != SAT_OK) return s;
-            if ((s = encode_map(&mo, SAT_INT32, dst, rows, cols, pitch, v.TR, v.TC)) != SAT_OK) return s;
+            if ((s = encode_map(&mo, SAT_INT32, dst, rows, cols, pitch, v.OBR, v.TC)) != SAT_OK) return s;
         } else {
             if ((s = encode_map(&mi, static_cast<sat_dtype_t>(dt), src, rows, cols, pitch, v.TR, v.TC)) != SAT_OK)
                 return s;
-            if ((s = encode_map(&mo, static_cast<sat_dtype_t>(dt), dst, rows, cols, pitch, v.TR, v.TC)) != SAT_OK)
+            if ((s = encode_map(&mo, static_cast<sat_dtype_t>(dt), dst, rows, cols, pitch, v.OBR, v.TC)) != SAT_OK)
                 return s;
         }
     }
@@ -570,7 +579,8 @@ sat_status_t colsum_impl(sat_dtype_t dt, const void* src, void* colsum, int64_t 
     DeviceInfo* di;
     sat_status_t s = device_info(dev, &di);
     if (s != SAT_OK) return s;
-    const int64_t bx = (cols + 255) / 256;
+    const bool vec = ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) && (pitch % 4 == 0);
+    const int64_t bx = (cols + (vec ? 1023 : 255)) / (vec ? 1024 : 256);
     int64_t nseg = (static_cast<int64_t>(di->sms) * 8 + bx - 1) / bx;
     const int64_t max_seg = (rows + 7) / 8;
     if (nseg > max_seg) nseg = max_seg;
@@ -584,13 +594,21 @@ sat_status_t colsum_impl(sat_dtype_t dt, const void* src, void* colsum, int64_t 
     if ((s = get_scratch(w, static_cast<size_t>(nseg * cols) * 4, &partial)) != SAT_OK) return s;
     dim3 g1(static_cast<unsigned>(bx), static_cast<unsigned>(nseg));
     if (dt == SAT_INT32) {
-        sat::colsum_partial_kernel<uint32_t><<<g1, 256, 0, st>>>(static_cast<const uint32_t*>(src),
-                                                                 static_cast<uint32_t*>(partial), rows, cols, pitch, seg);
+        if (vec)
+            sat::colsum_partial_kernel<uint32_t, true><<<g1, 256, 0, st>>>(
+                static_cast<const uint32_t*>(src), static_cast<uint32_t*>(partial), rows, cols, pitch, seg);
+        else
+            sat::colsum_partial_kernel<uint32_t, false><<<g1, 256, 0, st>>>(
+                static_cast<const uint32_t*>(src), static_cast<uint32_t*>(partial), rows, cols, pitch, seg);
         sat::colsum_reduce_kernel<uint32_t><<<static_cast<unsigned>((cols + 255) / 256), 256, 0, st>>>(
             static_cast<const uint32_t*>(partial), static_cast<uint32_t*>(colsum), cols, static_cast<int>(nseg));
     } else {
-        sat::colsum_partial_kernel<float><<<g1, 256, 0, st>>>(static_cast<const float*>(src),
-                                                              static_cast<float*>(partial), rows, cols, pitch, seg);
+        if (vec)
+            sat::colsum_partial_kernel<float, true><<<g1, 256, 0, st>>>(
+                static_cast<const float*>(src), static_cast<float*>(partial), rows, cols, pitch, seg);
+        else
+            sat::colsum_partial_kernel<float, false><<<g1, 256, 0, st>>>(
+                static_cast<const float*>(src), static_cast<float*>(partial), rows, cols, pitch, seg);
         sat::colsum_reduce_kernel<float><<<static_cast<unsigned>((cols + 255) / 256), 256, 0, st>>>(
             static_cast<const float*>(partial), static_cast<float*>(colsum), cols, static_cast<int>(nseg));
     }

@@ -7,30 +7,71 @@
 namespace sat {
 
 // Partial column sums: block (x, y) sums rows [y*seg, min((y+1)*seg, rows)) of columns
-// [x*256, x*256+256) into partial[y][col].  One thread per column: every warp reads 128 contiguous
-// bytes per row (coalesced); 8 independent rows in flight per thread.
-template <typename V>
+// [x*256*W, (x+1)*256*W) into partial[y][col], W = 4 columns per thread with 16-byte loads (VEC) or
+// 1 with 4-byte loads.  Every warp reads 512 (128) contiguous bytes per row; 8 independent rows in
+// flight per thread.  Per column: 8 row-residue accumulators, summed in ascending order at the end.
+template <typename V, bool VEC>
 __global__ void __launch_bounds__(256) colsum_partial_kernel(const V* __restrict__ src, V* __restrict__ partial,
                                                               int64_t rows, int64_t cols, int64_t pitch,
                                                               int64_t seg) {
-    const int64_t j = static_cast<int64_t>(blockIdx.x) * 256 + threadIdx.x;
+    constexpr int W = VEC ? 4 : 1;
+    const int64_t j = (static_cast<int64_t>(blockIdx.x) * 256 + threadIdx.x) * W;
     if (j >= cols) return;
     const int64_t r0 = static_cast<int64_t>(blockIdx.y) * seg;
     int64_t r1 = r0 + seg;
     if (r1 > rows) r1 = rows;
-    V acc[8];
+    V acc[8][W];
 #pragma unroll
-    for (int u = 0; u < 8; ++u) acc[u] = V(0);
+    for (int u = 0; u < 8; ++u)
+#pragma unroll
+        for (int c = 0; c < W; ++c) acc[u][c] = V(0);
+    const bool full = j + W <= cols;
     int64_t i = r0;
-    for (; i + 8 <= r1; i += 8) {
+    if (VEC && full) {
+        for (; i + 8 <= r1; i += 8) {
+            uint4 q[8];
 #pragma unroll
-        for (int u = 0; u < 8; ++u) acc[u] = acc[u] + __ldcs(src + (i + u) * pitch + j);
+            for (int u = 0; u < 8; ++u) q[u] = __ldcs(reinterpret_cast<const uint4*>(src + (i + u) * pitch + j));
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+                acc[u][0] = acc[u][0] + from_bits<V>(q[u].x);
+                if constexpr (W == 4) {
+                    acc[u][1] = acc[u][1] + from_bits<V>(q[u].y);
+                    acc[u][2] = acc[u][2] + from_bits<V>(q[u].z);
+                    acc[u][3] = acc[u][3] + from_bits<V>(q[u].w);
+                }
+            }
+        }
+        for (; i < r1; ++i) {
+            const uint4 q = __ldcs(reinterpret_cast<const uint4*>(src + i * pitch + j));
+            acc[0][0] = acc[0][0] + from_bits<V>(q.x);
+            if constexpr (W == 4) {
+                acc[0][1] = acc[0][1] + from_bits<V>(q.y);
+                acc[0][2] = acc[0][2] + from_bits<V>(q.z);
+                acc[0][3] = acc[0][3] + from_bits<V>(q.w);
+            }
+        }
+    } else {
+        for (; i + 8 <= r1; i += 8) {
+#pragma unroll
+            for (int u = 0; u < 8; ++u)
+#pragma unroll
+                for (int c = 0; c < W; ++c)
+                    if (j + c < cols) acc[u][c] = acc[u][c] + __ldcs(src + (i + u) * pitch + j + c);
+        }
+        for (; i < r1; ++i)
+#pragma unroll
+            for (int c = 0; c < W; ++c)
+                if (j + c < cols) acc[0][c] = acc[0][c] + __ldcs(src + i * pitch + j + c);
     }
-    for (; i < r1; ++i) acc[0] = acc[0] + __ldcs(src + i * pitch + j);
-    V tot = V(0);
 #pragma unroll
-    for (int u = 0; u < 8; ++u) tot = tot + acc[u];
-    partial[static_cast<int64_t>(blockIdx.y) * cols + j] = tot;
+    for (int c = 0; c < W; ++c) {
+        if (j + c >= cols) break;
+        V tot = V(0);
+#pragma unroll
+        for (int u = 0; u < 8; ++u) tot = tot + acc[u][c];
+        partial[static_cast<int64_t>(blockIdx.y) * cols + j + c] = tot;
+    }
 }
 
 // colsum[j] = sum over segments y = 0, 1, ... of partial[y][j] (ascending y).

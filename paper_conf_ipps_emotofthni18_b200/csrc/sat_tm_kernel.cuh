@@ -26,7 +26,7 @@
 
 namespace sat {
 
-template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0>
+template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0, int QS_ = 0>
 struct TmCfg {
     static constexpr int TR = 128, TC = 128, NW = NW_;
     static constexpr int IN = IN_;    // input stages
@@ -41,6 +41,8 @@ struct TmCfg {
     static constexpr int NREG = RPW * 4;         // 32-bit registers per thread parked per tile
     static constexpr int D = D_;                 // TMEM parking depth: finish(k) runs after local(k + D - 1)
     static constexpr bool DIRECT = DIRECT_ != 0; // GSAT stored from registers (st.global.cs), no output buffer
+    static constexpr bool QS = QS_ != 0;         // output buffer handed over in quarters (4 TMA stores of TR/4 rows)
+    static constexpr int OBR = QS ? TR / 4 : TR; // rows per TMA store box
     static constexpr int TM_COLS_PER_SLOT = (NW / 4) * NREG;
     static constexpr int TM_COLS = D * TM_COLS_PER_SLOT <= 32 ? 32 : D * TM_COLS_PER_SLOT <= 64 ? 64
                                  : D * TM_COLS_PER_SLOT <= 128 ? 128 : D * TM_COLS_PER_SLOT <= 256 ? 256 : 512;
@@ -74,7 +76,8 @@ struct TmSmem {
     uint64_t result[Cfg::NQ];  // GSAT of the slot's tile is in `out` (NW arrivals)
     uint64_t full[Cfg::IN];
     uint64_t empty[Cfg::IN];   // input stage read into registers (NW arrivals)
-    uint64_t ofree;            // `out` read by the TMA store
+    uint64_t ofree[4];         // quarter q of `out` read by its TMA store (only [0] without QS: the whole buffer)
+    uint64_t qready[4];        // QS: quarter q of `out` written (NW/4 arrivals)
     alignas(16) TileInfo info[Cfg::NQ];
     uint32_t epoch;
     int end_n;
@@ -216,6 +219,12 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
                 for (int r = 0; r < RPW; ++r) v[r][c] = V(0);
             }
     }
+#if SAT_STATS
+    const bool skip = (p.order & 64) != 0;  // timing experiment only: no local SAT / publication (wrong sums)
+#else
+    constexpr bool skip = false;
+#endif
+    if (!skip) {
     // local SAT: column prefix in the band, warp prefix-sum rows, bands above
 #pragma unroll
     for (int r = 1; r < RPW; ++r)
@@ -309,6 +318,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
                 }
             }
         }
+    }
     }
     // park the block
     uint32_t r32[Cfg::NREG];
@@ -413,8 +423,10 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
                        make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3])));
         }
     } else if (!ragged) {
+        constexpr int WPQ = NW / 4;  // warps per quarter of the buffer
+        const int qq = Cfg::QS ? warp / WPQ : 0;
         SAT_CLK(o0);
-        mbar_wait(&sm.ofree, (ou & 1u) ^ 1u);  // the previous tile's store has read `out`
+        mbar_wait(&sm.ofree[qq], (ou & 1u) ^ 1u);  // the previous tile's store has read (this quarter of) `out`
         SAT_CLK(o1);
         if (warp == 0 && lane == 0) WS_ST(kWsFastHits, o1 - o0);
 #pragma unroll
@@ -422,6 +434,10 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
             *reinterpret_cast<uint4*>(&sm.out[(row0 + r) * TC + col0]) =
                 make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3]));
         fence_proxy_async_smem();
+        if constexpr (Cfg::QS) {
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&sm.qready[qq]);
+        }
     } else {
 #pragma unroll
         for (int r = 0; r < RPW; ++r) {
@@ -620,7 +636,10 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
             mbar_init(&sm.full[s], 1);
             mbar_init(&sm.empty[s], NW);
         }
-        mbar_init(&sm.ofree, 1);
+        for (int q = 0; q < 4; ++q) {
+            mbar_init(&sm.ofree[q], 1);
+            mbar_init(&sm.qready[q], NW / 4);
+        }
         fence_mbar_init();
     }
     tc_fence_before();
@@ -668,11 +687,32 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         if (lane == 0) {
             if constexpr (TMA) prefetch_tensormap(&map_out);
             const uint64_t spol = policy_evict_first();
+            uint32_t sou = 0;  // QS: uses of the output buffer so far
             for (Slot<Cfg::NQ> tq;; tq.next()) {
                 mbar_wait(&sm.acq[tq.s], tq.ph);
                 const TileInfo ti = sm.info[tq.s];
                 if (ti.t >= p.ntiles) break;
                 SAT_CLK(u0);
+                if constexpr (Cfg::QS && !Cfg::DIRECT) {
+                    // quarters go out as soon as their warps have written them
+                    const bool qragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
+                    if (!qragged) {
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            mbar_wait(&sm.qready[q], sou & 1u);
+                            tma_store_2d_hint(&map_out, sm.out + q * Cfg::OBR * TC, ti.J * TC, ti.I * TR + q * Cfg::OBR,
+                                              spol);
+                            bulk_commit();
+                            if (q > 0) {
+                                bulk_wait_read<1>();
+                                mbar_arrive(&sm.ofree[q - 1]);
+                            }
+                        }
+                        bulk_wait_read<0>();
+                        mbar_arrive(&sm.ofree[3]);
+                        ++sou;
+                    }
+                }
                 mbar_wait(&sm.result[tq.s], tq.ph);
                 // tile k is done with its slot (walks, carries, id): tile k + NQ may be acquired.  Released
                 // only here so that no barrier of the slot can run a phase ahead of this lane.
@@ -680,14 +720,14 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 SAT_CLK(u1);
                 WS_ST(kWsStResultWait, u1 - u0);
                 const bool ragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
-                if (!Cfg::DIRECT && !ragged) {
+                if (!Cfg::DIRECT && !Cfg::QS && !ragged) {
                     tma_store_2d_hint(&map_out, sm.out, ti.J * TC, ti.I * TR, spol);
                     bulk_commit();
 #if SAT_STATS
                     if (p.trace) p.trace[8LL * ti.t + 6] = static_cast<long long>(globaltimer_ns());
 #endif
                     bulk_wait_read<0>();
-                    mbar_arrive(&sm.ofree);
+                    mbar_arrive(&sm.ofree[0]);
                 }
                 SAT_CLK(u2);
                 WS_ST(kWsStStore, u2 - u1);
