@@ -63,6 +63,7 @@ using PrepareFn = cudaError_t (*)(bool tma, bool carry, int* occupancy);
 
 struct Variant {
     int TR, TC, NW, STAGES;
+    int TB;                // TMA box width in elements (TC, or 256 for flat tiles: NB = TC / TB boxes)
     int OBR;               // rows of the output TMA box (TR, or TR/4 for quarter stores)
     int family;            // 2 = TMEM-parked (sat_tm_kernel), 1 = warp-specialised (sat_ws_kernel), 0 = classic
     size_t smem;           // dynamic shared memory bytes (same for int32 / fp32)
@@ -97,9 +98,10 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
 };
 
-template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS>
-struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS>> {
-    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS>;
+template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC>;
+    static constexpr int box_cols = Cfg::TB;
     static constexpr int out_box_rows = Cfg::OBR;
     static constexpr int threads = Cfg::THREADS;
     static constexpr int family = 2;
@@ -117,6 +119,11 @@ template <typename F, typename = void>
 struct HasOBR { static constexpr bool value = false; };
 template <typename F>
 struct HasOBR<F, std::void_t<decltype(F::out_box_rows)>> { static constexpr bool value = true; };
+
+template <typename F, typename = void>
+struct HasBox { static constexpr bool value = false; };
+template <typename F>
+struct HasBox<F, std::void_t<decltype(F::box_cols)>> { static constexpr bool value = true; };
 
 template <typename F, typename = void>
 struct HasU8 { static constexpr bool value = false; };
@@ -190,7 +197,9 @@ Variant make_variant() {
     v.launch[SAT_FLOAT32] = &launch_variant<float, Cfg>;
     v.prepare[SAT_INT32] = &prepare_variant<uint32_t, Cfg>;
     v.prepare[SAT_FLOAT32] = &prepare_variant<float, Cfg>;
-    if constexpr (HasU8<Family<Cfg>>::value) {
+    if constexpr (HasBox<Family<Cfg>>::value) v.TB = Family<Cfg>::box_cols;
+    else v.TB = Cfg::TC;
+    if constexpr (HasU8<Family<Cfg>>::value && Cfg::TC == 128) {
         v.launch[kU8] = &launch_variant_u8<Cfg>;
         v.prepare[kU8] = &prepare_variant_u8<Cfg>;
     } else {
@@ -213,6 +222,9 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 8
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),  // 9
         make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>>(),  // 10: u8 integral images only (4 stages of 16 KiB u8 tiles)
+        make_variant<sat::TmCfg<8, 2, 5, 1, 3, 4, 0, 0, 32, 512>>(),   // 11: flat 32 x 512 tiles, 8 compute warps
+        make_variant<sat::TmCfg<16, 2, 5, 1, 3, 4, 0, 0, 64, 256>>(),  // 12: flat 64 x 256 tiles
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),   // 13: flat 64 x 256 tiles, 8 compute warps
     };
     return vs;
 }
@@ -513,9 +525,9 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
             if ((s = encode_map_u8(&mi, src, rows, cols, src_pitch, v.TR, v.TC)) != SAT_OK) return s;
             if ((s = encode_map(&mo, SAT_INT32, dst, rows, cols, pitch, v.OBR, v.TC)) != SAT_OK) return s;
         } else {
-            if ((s = encode_map(&mi, static_cast<sat_dtype_t>(dt), src, rows, cols, pitch, v.TR, v.TC)) != SAT_OK)
+            if ((s = encode_map(&mi, static_cast<sat_dtype_t>(dt), src, rows, cols, pitch, v.TR, v.TB)) != SAT_OK)
                 return s;
-            if ((s = encode_map(&mo, static_cast<sat_dtype_t>(dt), dst, rows, cols, pitch, v.OBR, v.TC)) != SAT_OK)
+            if ((s = encode_map(&mo, static_cast<sat_dtype_t>(dt), dst, rows, cols, pitch, v.OBR, v.TB)) != SAT_OK)
                 return s;
         }
     }
@@ -652,6 +664,21 @@ sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, in
     if (gy > 65535) gy = 65535;
     const dim3 grid(static_cast<unsigned>(gx), static_cast<unsigned>(gy));
     const bool vec = ((reinterpret_cast<uintptr_t>(out) & 15u) == 0) && ((pitch * 4) % 16 == 0);
+    // staged kernel: both pointers 16-byte aligned and the two double-buffered row segments in 48 KB
+    const int64_t nv = (sat::kBoxPanel + 2 * rw + 8) / 4 + 1;
+    const size_t smem = static_cast<size_t>(nv) * 4 * 4 * 4;
+    if (vec && ((reinterpret_cast<uintptr_t>(b) & 15u) == 0) && smem <= 48 * 1024) {
+        if (dt == SAT_INT32)
+            sat::box_sum_smem_kernel<uint32_t><<<grid, sat::kBoxThreads, smem, st>>>(
+                static_cast<const uint32_t*>(b), static_cast<uint32_t*>(out), rows, cols, pitch, rh, rw,
+                static_cast<int>(nv));
+        else
+            sat::box_sum_smem_kernel<float><<<grid, sat::kBoxThreads, smem, st>>>(
+                static_cast<const float*>(b), static_cast<float*>(out), rows, cols, pitch, rh, rw, static_cast<int>(nv));
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return cuda_fail(e, "box_sum_smem_kernel");
+        return SAT_OK;
+    }
     if (dt == SAT_INT32) {
         const uint32_t* bb = static_cast<const uint32_t*>(b);
         uint32_t* oo = static_cast<uint32_t*>(out);

@@ -59,6 +59,77 @@ __global__ void __launch_bounds__(256) box_sum_kernel(const V* __restrict__ b, V
     }
 }
 
+// Staged box filter (the production path when the two row segments fit in shared memory).  A block
+// owns a panel of kBoxPanel output columns and walks output rows i = blockIdx.y, +gridDim.y, ...  Per
+// row it copies the two SAT row segments the panel needs, rows d and u over columns
+// [panel - rw - 1, panel + kBoxPanel - 1 + rw] (clipped to the matrix; index -1 and the rows above
+// row 0 read as zero), into shared memory with 16-byte coalesced loads, then evaluates P:48 for
+// its 4 columns (256 apart, so a warp reads consecutive shared-memory words) from shared memory in
+// the same left-to-right order as box_sum_kernel.  Global traffic per
+// output row: one read of each SAT row segment (row u is row d of the output row 2*rh+1 above, an L2
+// hit) and coalesced streaming stores, instead of 16 scalar L2 loads per 4 outputs.
+// Requires pitch * 4 and both pointers 16-byte aligned (VEC).  Double-buffered: the segments of the
+// next row are loaded while the current row is evaluated.
+constexpr int kBoxThreads = 256;
+constexpr int kBoxPanel = 4 * kBoxThreads;
+
+template <typename V>
+__device__ __forceinline__ void box_load_seg(const V* __restrict__ b, int64_t pitch, int64_t row, int64_t a0,
+                                             int64_t hi, int nv, V* seg) {
+    // seg[k] = b[row][a0 + k] for a0 + k in [0, hi], else 0 (a0 is a multiple of 4; hi = last column)
+    for (int q = threadIdx.x; q < nv; q += blockDim.x) {
+        const int64_t j = a0 + 4 * static_cast<int64_t>(q);
+        uint4 w = make_uint4(0u, 0u, 0u, 0u);
+        if (row >= 0 && j >= 0 && j <= hi) w = __ldcg(reinterpret_cast<const uint4*>(b + row * pitch + j));
+        if (row >= 0 && j + 3 > hi) {  // columns past the last one read as zero (within the pitch row)
+            if (j + 1 > hi) w.y = 0u;
+            if (j + 2 > hi) w.z = 0u;
+            if (j + 3 > hi) w.w = 0u;
+            if (j > hi) w.x = 0u;
+        }
+        *reinterpret_cast<uint4*>(seg + 4 * q) = w;
+    }
+}
+
+template <typename V>
+__global__ void __launch_bounds__(kBoxThreads) box_sum_smem_kernel(const V* __restrict__ b, V* __restrict__ out,
+                                                                   int64_t rows, int64_t cols, int64_t pitch,
+                                                                   int64_t rh, int64_t rw, int nv) {
+    extern __shared__ __align__(16) unsigned char box_smem[];
+    V* buf = reinterpret_cast<V*>(box_smem);  // [2 buffers][2 rows (d, u)][4 * nv]
+    const int64_t p0 = static_cast<int64_t>(blockIdx.x) * kBoxPanel;
+    const int64_t a0 = ((p0 - rw - 1) >= 0) ? ((p0 - rw - 1) & ~int64_t(3)) : -((-(p0 - rw - 1) + 3) & ~int64_t(3));
+    const int64_t hi = cols - 1;
+    const int seglen = 4 * nv;
+    auto load_row = [&](int64_t i, int sb) {
+        const int64_t u = i - rh - 1;
+        const int64_t d = i + rh < rows - 1 ? i + rh : rows - 1;
+        box_load_seg(b, pitch, d, a0, hi, nv, buf + (2 * sb) * seglen);
+        box_load_seg(b, pitch, u, a0, hi, nv, buf + (2 * sb + 1) * seglen);
+    };
+    int sb = 0;
+    int64_t i = blockIdx.y;
+    if (i < rows) load_row(i, 0);
+    for (; i < rows; i += gridDim.y) {
+        __syncthreads();  // segments of row i are in buffer sb; buffer sb^1 is free
+        if (i + gridDim.y < rows) load_row(i + gridDim.y, sb ^ 1);
+        const V* D = buf + (2 * sb) * seglen;
+        const V* U = D + seglen;
+        V* dst = out + i * pitch;
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {  // column p0 + threadIdx.x + 256 c: a warp reads consecutive words
+            const int64_t j = p0 + threadIdx.x + kBoxThreads * c;
+            if (j < cols) {
+                const int64_t l = j - rw - 1;
+                const int64_t r = j + rw < hi ? j + rw : hi;
+                const int kr = static_cast<int>(r - a0), kl = static_cast<int>(l - a0);
+                __stcs(dst + j, ((D[kr] - U[kr]) - D[kl]) + U[kl]);
+            }
+        }
+        sb ^= 1;
+    }
+}
+
 // Batched rectangle queries: rects[k] = (u, d, l, r) in the convention of P:48 (u < i <= d,
 // l < j <= r).  Indices are clamped into [-1, rows-1] / [-1, cols-1] (memory safety); an empty
 // rectangle (u >= d or l >= r after clamping) gives 0.

@@ -26,9 +26,16 @@
 
 namespace sat {
 
-template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0, int QS_ = 0>
+// TR_ x TC_ tiles: TC_ = 128 * G (a lane owns G chunks of 4 columns, 128 apart); flat tiles (TC_ > 128)
+// keep the tile's 64 KiB but make every DRAM row visit 4 B * TC_ long (tile shape).
+template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0, int QS_ = 0,
+          int TR_ = 128, int TC_ = 128>
 struct TmCfg {
-    static constexpr int TR = 128, TC = 128, NW = NW_;
+    static constexpr int TR = TR_, TC = TC_, NW = NW_;
+    static constexpr int G = TC / 128;             // column chunks per lane
+    static constexpr int TB = TC < 256 ? TC : 256;  // TMA box width (boxDim <= 256 elements)
+    static constexpr int NB = TC / TB;              // TMA boxes per tile (stage / output layout [NB][TR][TB])
+    static constexpr bool SBAND = TC > 128;         // band bottoms exchanged through the tile's input stage
     static constexpr int IN = IN_;    // input stages
     static constexpr int STAGES = IN;
     static constexpr int NQ = NQ_;    // tile ring
@@ -38,7 +45,7 @@ struct TmCfg {
     static constexpr bool WPUB_WAIT = WPUB_ == 2;  // ... blocking on the tile's local aggregates
     static constexpr bool DECOUPLED = WPUB_ == 3;  // tm_walker: GLS published as a local corner word
     static constexpr int RPW = TR / NW, ER = TR / 32, EC = TC / 32;
-    static constexpr int NREG = RPW * 4;         // 32-bit registers per thread parked per tile
+    static constexpr int NREG = RPW * 4 * G;     // 32-bit registers per thread parked per tile
     static constexpr int D = D_;                 // TMEM parking depth: finish(k) runs after local(k + D - 1)
     static constexpr bool DIRECT = DIRECT_ != 0; // GSAT stored from registers (st.global.cs), no output buffer
     static constexpr bool QS = QS_ != 0;         // output buffer handed over in quarters (4 TMA stores of TR/4 rows)
@@ -49,7 +56,9 @@ struct TmCfg {
     static constexpr int ROW_WARP = NW, COL_WARP = NW + 1, STORE_WARP = NW + 2, LOAD_WARP = NW + 3;
     static constexpr int THREADS = (NW + 4) * 32;
     static_assert(NW % 4 == 0 && TR % NW == 0 && RPW % 4 == 0, "compute warps cover the 4 TMEM lane quarters");
-    static_assert(NREG == 16 || NREG == 32, "tcgen05 32x32b.x16 / .x32 parking");
+    static_assert(NREG == 16 || NREG == 32 || NREG == 64, "tcgen05 32x32b.x16 / .x32 parking");
+    static_assert(TC % 128 == 0 && TC % TB == 0 && TR >= 32 && TR * TC == 128 * 128, "64 KiB tiles, TC = 128 G");
+    static_assert(!SBAND || (NW <= TR && !DIRECT && !QS), "flat tiles: band rows fit in a stage, TMA stores");
     static_assert(D >= 2 && D * TM_COLS_PER_SLOT <= 512, "TMEM columns");
     static_assert(IN >= 1 && NQ >= IN + D - 1 && NQ <= 16, "rings");
 };
@@ -58,7 +67,7 @@ template <typename V, typename Cfg, typename TIn = V>
 struct TmSmem {
     alignas(1024) TIn stage[Cfg::IN][Cfg::TR * Cfg::TC];  // input ring (TMA loads; u8 for integral images)
     alignas(1024) V out[Cfg::DIRECT ? 4 : Cfg::TR * Cfg::TC];  // GSAT of one tile (TMA store source)
-    alignas(16) V band[2][Cfg::NW][Cfg::TC];
+    alignas(16) V band[Cfg::SBAND ? 1 : 2][Cfg::SBAND ? 1 : Cfg::NW][Cfg::SBAND ? 4 : Cfg::TC];
     alignas(16) V rp[Cfg::NQ][Cfg::TR];
     alignas(16) V cp[Cfg::NQ][Cfg::TC];
     V corner[Cfg::NQ];
@@ -157,14 +166,40 @@ __device__ __forceinline__ uint32_t tm_addr(uint32_t base, int warp, int slot) {
            static_cast<uint32_t>(slot * Cfg::TM_COLS_PER_SLOT + (warp >> 2) * Cfg::NREG);
 }
 
+// Element (r, c) of a stage / the output buffer: NB boxes of TR x TB, each row-major.
+template <typename Cfg>
+__device__ __forceinline__ constexpr int tm_sidx(int r, int c) {
+    return (c / Cfg::TB) * (Cfg::TR * Cfg::TB) + r * Cfg::TB + (c % Cfg::TB);
+}
+
+template <int N>
+__device__ __forceinline__ void tmem_st_blk(uint32_t taddr, const uint32_t (&r)[N]) {
+    if constexpr (N == 64) {
+        tmem_st<32>(taddr, *reinterpret_cast<const uint32_t(*)[32]>(&r[0]));
+        tmem_st<32>(taddr + 32, *reinterpret_cast<const uint32_t(*)[32]>(&r[32]));
+    } else {
+        tmem_st<N>(taddr, r);
+    }
+}
+template <int N>
+__device__ __forceinline__ void tmem_ld_blk(uint32_t taddr, uint32_t (&r)[N]) {
+    if constexpr (N == 64) {
+        tmem_ld<32>(taddr, *reinterpret_cast<uint32_t(*)[32]>(&r[0]));
+        tmem_ld<32>(taddr + 32, *reinterpret_cast<uint32_t(*)[32]>(&r[32]));
+    } else {
+        tmem_ld<N>(taddr, r);
+    }
+}
+
 // Step 1 + local SAT + Steps 2.A.1 / 2.B.1 of tile k (input stage sl, tile slot tq); parks the block in
 // TMEM slot k % D.  Returns false at the end marker.
 template <typename V, typename Cfg, bool TMA, typename TIn>
 __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, const Slot<Cfg::IN>& sl,
                                          const Slot<Cfg::NQ>& tq, uint32_t epoch, int warp, int lane) {
-    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW, G = Cfg::G, X = 4 * Cfg::G;
+    static_assert(sizeof(TIn) != 1 || TC == 128, "u8 tiles: 128 columns");
     const int s = sl.s;
-    const int row0 = warp * RPW, col0 = lane * 4;
+    const int row0 = warp * RPW, col0 = lane * 4;  // this lane's columns: g * 128 + col0 + c
     SAT_CLK(c0);
     mbar_wait(&sm.full[s], sl.ph);
     SAT_CLK(c1);
@@ -177,7 +212,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
     const int I = ti.I, J = ti.J;
     const long long tidx = static_cast<long long>(I) * p.C + J;
     const int par = tq.k & 1;
-    V v[RPW][4];
+    V v[RPW][X];
     if constexpr (TMA && sizeof(TIn) == 1) {
         // u8 pixels (integral image): a lane's 4 columns are one 32-bit word of the stage row
         const TIn* tile = sm.stage[s];
@@ -190,33 +225,38 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
     } else if constexpr (TMA) {
         const TIn* tile = sm.stage[s];
 #pragma unroll
-        for (int r = 0; r < RPW; ++r) {
-            const uint4 q = *reinterpret_cast<const uint4*>(&tile[(row0 + r) * TC + col0]);
-            v[r][0] = from_bits<V>(q.x); v[r][1] = from_bits<V>(q.y);
-            v[r][2] = from_bits<V>(q.z); v[r][3] = from_bits<V>(q.w);
-        }
+        for (int r = 0; r < RPW; ++r)
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                const uint4 q = *reinterpret_cast<const uint4*>(&tile[tm_sidx<Cfg>(row0 + r, g * 128 + col0)]);
+                v[r][4 * g] = from_bits<V>(q.x); v[r][4 * g + 1] = from_bits<V>(q.y);
+                v[r][4 * g + 2] = from_bits<V>(q.z); v[r][4 * g + 3] = from_bits<V>(q.w);
+            }
     } else {
 #pragma unroll
         for (int r = 0; r < RPW; ++r) {
             const long long gi = static_cast<long long>(I) * TR + row0 + r;
 #pragma unroll
-            for (int c = 0; c < 4; ++c) {
-                const long long gj = static_cast<long long>(J) * TC + col0 + c;
+            for (int x = 0; x < X; ++x) {
+                const long long gj = static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4);
                 const bool in = gi < p.rows && gj < p.cols;
-                if constexpr (sizeof(TIn) == 1) v[r][c] = in ? V(p.src8[gi * p.src_pitch + gj]) : V(0);
-                else v[r][c] = in ? p.src[gi * p.pitch + gj] : V(0);
+                if constexpr (sizeof(TIn) == 1) v[r][x] = in ? V(p.src8[gi * p.src_pitch + gj]) : V(0);
+                else v[r][x] = in ? p.src[gi * p.pitch + gj] : V(0);
             }
         }
     }
-    // the pixels are in registers: the loader may refill the stage now
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&sm.empty[s]);
+    // the pixels are in registers: the loader may refill the stage now (flat tiles: after the band
+    // exchange, which goes through this stage)
+    if constexpr (!Cfg::SBAND) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.empty[s]);
+    }
     if (TMA && J == p.C - 1) {  // right edge: zero columns >= cols (16-byte TMA granules, reading R2)
 #pragma unroll
-        for (int c = 0; c < 4; ++c)
-            if (static_cast<long long>(J) * TC + col0 + c >= p.cols) {
+        for (int x = 0; x < X; ++x)
+            if (static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4) >= p.cols) {
 #pragma unroll
-                for (int r = 0; r < RPW; ++r) v[r][c] = V(0);
+                for (int r = 0; r < RPW; ++r) v[r][x] = V(0);
             }
     }
 #if SAT_STATS
@@ -229,33 +269,67 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
 #pragma unroll
     for (int r = 1; r < RPW; ++r)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + v[r - 1][c];
+        for (int x = 0; x < X; ++x) v[r][x] = v[r][x] + v[r - 1][x];
 #pragma unroll
     for (int r = 0; r < RPW; ++r) {
-        v[r][1] = v[r][1] + v[r][0];
-        v[r][2] = v[r][2] + v[r][1];
-        v[r][3] = v[r][3] + v[r][2];
-        const V incl = warp_inclusive_scan(v[r][3], lane);
-        V excl = __shfl_up_sync(kFull, incl, 1);
-        if (lane == 0) excl = V(0);
+        V carry = V(0);  // row total of the chunks to the left
 #pragma unroll
-        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + excl;
+        for (int g = 0; g < G; ++g) {
+            V* w = &v[r][4 * g];
+            w[1] = w[1] + w[0];
+            w[2] = w[2] + w[1];
+            w[3] = w[3] + w[2];
+            const V incl = warp_inclusive_scan(w[3], lane);
+            V excl = __shfl_up_sync(kFull, incl, 1);
+            if (lane == 0) excl = V(0);
+            if (g > 0) excl = excl + carry;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) w[c] = w[c] + excl;
+            if (g + 1 < G) carry = carry + __shfl_sync(kFull, incl, 31);
+        }
     }
-    *reinterpret_cast<uint4*>(&sm.band[par][warp][col0]) =
-        make_uint4(to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
-    named_bar_sync(1, NW * 32);
-    {   // band offsets: warp w adds the bottoms of bands 0 .. w-1 (one barrier, no serial scan)
-        V off[4] = {V(0), V(0), V(0), V(0)};
+    {   // band offsets: warp w adds the bottoms of bands 0 .. w-1 (no serial scan)
+        V off[X];
+#pragma unroll
+        for (int x = 0; x < X; ++x) off[x] = V(0);
+        if constexpr (Cfg::SBAND) {
+            // every warp has read its rows of the stage: the stage holds the band bottoms (row w at w * TC)
+            V* bands = reinterpret_cast<V*>(sm.stage[s]);
+            named_bar_sync(1, NW * 32);
+#pragma unroll
+            for (int g = 0; g < G; ++g)
+                *reinterpret_cast<uint4*>(&bands[warp * TC + g * 128 + col0]) =
+                    make_uint4(to_bits(v[RPW - 1][4 * g]), to_bits(v[RPW - 1][4 * g + 1]),
+                               to_bits(v[RPW - 1][4 * g + 2]), to_bits(v[RPW - 1][4 * g + 3]));
+            named_bar_sync(1, NW * 32);
+#pragma unroll 2
+            for (int u = 0; u < warp; ++u)
+#pragma unroll
+                for (int g = 0; g < G; ++g) {
+                    const uint4 q = *reinterpret_cast<const uint4*>(&bands[u * TC + g * 128 + col0]);
+                    off[4 * g] = off[4 * g] + from_bits<V>(q.x); off[4 * g + 1] = off[4 * g + 1] + from_bits<V>(q.y);
+                    off[4 * g + 2] = off[4 * g + 2] + from_bits<V>(q.z);
+                    off[4 * g + 3] = off[4 * g + 3] + from_bits<V>(q.w);
+                }
+            // generic-proxy writes to the stage precede the next TMA (async-proxy) write into it
+            fence_proxy_async_smem();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&sm.empty[s]);
+        } else {
+            *reinterpret_cast<uint4*>(&sm.band[par][warp][col0]) = make_uint4(
+                to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
+            named_bar_sync(1, NW * 32);
 #pragma unroll 4
-        for (int u = 0; u < warp; ++u) {
-            const uint4 q = *reinterpret_cast<const uint4*>(&sm.band[par][u][col0]);
-            off[0] = off[0] + from_bits<V>(q.x); off[1] = off[1] + from_bits<V>(q.y);
-            off[2] = off[2] + from_bits<V>(q.z); off[3] = off[3] + from_bits<V>(q.w);
+            for (int u = 0; u < warp; ++u) {
+                const uint4 q = *reinterpret_cast<const uint4*>(&sm.band[par][u][col0]);
+                off[0] = off[0] + from_bits<V>(q.x); off[1] = off[1] + from_bits<V>(q.y);
+                off[2] = off[2] + from_bits<V>(q.z); off[3] = off[3] + from_bits<V>(q.w);
+            }
         }
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
 #pragma unroll
-            for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + off[c];
+            for (int x = 0; x < X; ++x) v[r][x] = v[r][x] + off[x];
     }
     // Steps 2.A.1 / 2.B.1 (edge tiles publish inclusive at once: their carry is zero)
     const uint64_t pol = policy_evict_last();
@@ -264,25 +338,33 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
         const uint32_t kind = (J == 0) ? kIncl : kLocal;
 #pragma unroll
         for (int r = 0; r < RPW; r += 2)
-            st_relaxed2_p(rs + r, pack(epoch, kind, to_bits(v[r][3])), pack(epoch, kind, to_bits(v[r + 1][3])), pol);
+            st_relaxed2_p(rs + r, pack(epoch, kind, to_bits(v[r][X - 1])), pack(epoch, kind, to_bits(v[r + 1][X - 1])),
+                          pol);
     }
     if (warp == NW - 1) {
-        uint64_t* cs = p.col_slots + tidx * TC + col0;
         const uint32_t kind = (I == 0) ? kIncl : kLocal;
-        st_relaxed2_p(cs, pack(epoch, kind, to_bits(v[RPW - 1][0])), pack(epoch, kind, to_bits(v[RPW - 1][1])), pol);
-        st_relaxed2_p(cs + 2, pack(epoch, kind, to_bits(v[RPW - 1][2])), pack(epoch, kind, to_bits(v[RPW - 1][3])),
-                      pol);
+#pragma unroll
+        for (int g = 0; g < G; ++g) {
+            uint64_t* cs = p.col_slots + tidx * TC + g * 128 + col0;
+            const V* b = &v[RPW - 1][4 * g];
+            st_relaxed2_p(cs, pack(epoch, kind, to_bits(b[0])), pack(epoch, kind, to_bits(b[1])), pol);
+            st_relaxed2_p(cs + 2, pack(epoch, kind, to_bits(b[2])), pack(epoch, kind, to_bits(b[3])), pol);
+        }
     }
     if constexpr (Cfg::WPUB) {
         if (lane == 31) {
 #pragma unroll
             for (int r = 0; r < RPW; r += 4)
                 *reinterpret_cast<uint4*>(&sm.lrs[tq.s][row0 + r]) =
-                    make_uint4(to_bits(v[r][3]), to_bits(v[r + 1][3]), to_bits(v[r + 2][3]), to_bits(v[r + 3][3]));
+                    make_uint4(to_bits(v[r][X - 1]), to_bits(v[r + 1][X - 1]), to_bits(v[r + 2][X - 1]),
+                               to_bits(v[r + 3][X - 1]));
         }
         if (warp == NW - 1)
-            *reinterpret_cast<uint4*>(&sm.lcs[tq.s][col0]) = make_uint4(
-                to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
+#pragma unroll
+            for (int g = 0; g < G; ++g)
+                *reinterpret_cast<uint4*>(&sm.lcs[tq.s][g * 128 + col0]) =
+                    make_uint4(to_bits(v[RPW - 1][4 * g]), to_bits(v[RPW - 1][4 * g + 1]),
+                               to_bits(v[RPW - 1][4 * g + 2]), to_bits(v[RPW - 1][4 * g + 3]));
         __syncwarp();
         if (lane == 0) mbar_arrive(&sm.ldone[tq.s]);
         if constexpr (Cfg::DECOUPLED) {
@@ -295,38 +377,47 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
                 uint64_t* rs = p.row_slots + tidx * TR + row0;
 #pragma unroll
                 for (int r = 0; r < RPW; r += 2)
-                    st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + sm.rp[tq.s][row0 + r])),
-                                  pack(epoch, kIncl, to_bits(v[r + 1][3] + sm.rp[tq.s][row0 + r + 1])), pol);
+                    st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][X - 1] + sm.rp[tq.s][row0 + r])),
+                                  pack(epoch, kIncl, to_bits(v[r + 1][X - 1] + sm.rp[tq.s][row0 + r + 1])), pol);
             }
             if (warp == NW - 1) {
                 const int cd = __shfl_sync(kFull, *reinterpret_cast<volatile int*>(&sm.cdone[tq.s]), 0);
                 if (cd == tq.k + 1) {
                     __threadfence_block();
                     if (I > 0) {
-                        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[tq.s][col0]);
-                        uint64_t* cs = p.col_slots + tidx * TC + col0;
-                        st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + from_bits<V>(c4.x))),
-                                      pack(epoch, kIncl, to_bits(v[RPW - 1][1] + from_bits<V>(c4.y))), pol);
-                        st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + from_bits<V>(c4.z))),
-                                      pack(epoch, kIncl, to_bits(v[RPW - 1][3] + from_bits<V>(c4.w))), pol);
+#pragma unroll
+                        for (int g = 0; g < G; ++g) {
+                            const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[tq.s][g * 128 + col0]);
+                            uint64_t* cs = p.col_slots + tidx * TC + g * 128 + col0;
+                            const V* b = &v[RPW - 1][4 * g];
+                            st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(b[0] + from_bits<V>(c4.x))),
+                                          pack(epoch, kIncl, to_bits(b[1] + from_bits<V>(c4.y))), pol);
+                            st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(b[2] + from_bits<V>(c4.z))),
+                                          pack(epoch, kIncl, to_bits(b[3] + from_bits<V>(c4.w))), pol);
+                        }
                     }
                     if (lane == 31 && *reinterpret_cast<volatile int*>(&sm.rdone[tq.s]) == tq.k + 1) {
                         __threadfence_block();
-                        const V gs = sm.corner[tq.s] + ((v[RPW - 1][3] + sm.rp[tq.s][TR - 1]) + sm.cp[tq.s][TC - 1]);
+                        const V gs =
+                            sm.corner[tq.s] + ((v[RPW - 1][X - 1] + sm.rp[tq.s][TR - 1]) + sm.cp[tq.s][TC - 1]);
                         st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(gs)), pol);
                     }
                 }
             }
         }
     }
+    } else if constexpr (Cfg::SBAND) {
+        named_bar_sync(1, NW * 32);  // timing experiment: the stage may be refilled once every warp has read it
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&sm.empty[s]);
     }
     // park the block
     uint32_t r32[Cfg::NREG];
 #pragma unroll
     for (int r = 0; r < RPW; ++r)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) r32[r * 4 + c] = to_bits(v[r][c]);
-    tmem_st<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k % Cfg::D), r32);
+        for (int x = 0; x < X; ++x) r32[r * X + x] = to_bits(v[r][x]);
+    tmem_st_blk<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k % Cfg::D), r32);
     SAT_CLK(c2);
     if (warp == 0 && lane == 0) WS_ST(kWsLocal, c2 - c1);
 #if SAT_STATS
@@ -340,22 +431,22 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
 template <typename V, typename Cfg, bool TMA, bool CARRY, typename TIn>
 __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, const Slot<Cfg::NQ>& tq,
                                           uint32_t ou, uint32_t epoch, int warp, int lane) {
-    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW;
+    constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW, G = Cfg::G, X = 4 * Cfg::G;
     const int q = tq.s;
     const int row0 = warp * RPW, col0 = lane * 4;
     const TileInfo ti = sm.info[q];
     const int I = ti.I, J = ti.J;
     const long long tidx = static_cast<long long>(I) * p.C + J;
     const uint64_t pol = policy_evict_last();
-    V v[RPW][4];
+    V v[RPW][X];
     {
         uint32_t r32[Cfg::NREG];
         tmem_st_wait();
-        tmem_ld<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k % Cfg::D), r32);
+        tmem_ld_blk<Cfg::NREG>(tm_addr<Cfg>(sm.tmem_base, warp, tq.k % Cfg::D), r32);
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
 #pragma unroll
-            for (int c = 0; c < 4; ++c) v[r][c] = from_bits<V>(r32[r * 4 + c]);
+            for (int x = 0; x < X; ++x) v[r][x] = from_bits<V>(r32[r * X + x]);
     }
     SAT_CLK(c0);
     mbar_wait(&sm.rowwalk[q], tq.ph);
@@ -369,47 +460,53 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
         rt[r] = from_bits<V>(u.x); rt[r + 1] = from_bits<V>(u.y); rt[r + 2] = from_bits<V>(u.z);
         rt[r + 3] = from_bits<V>(u.w);
     }
-    V cpv[4];
-    {
-        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[q][col0]);
-        cpv[0] = from_bits<V>(c4.x); cpv[1] = from_bits<V>(c4.y); cpv[2] = from_bits<V>(c4.z);
-        cpv[3] = from_bits<V>(c4.w);
+    V cpv[X];
+#pragma unroll
+    for (int g = 0; g < G; ++g) {
+        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[q][g * 128 + col0]);
+        cpv[4 * g] = from_bits<V>(c4.x); cpv[4 * g + 1] = from_bits<V>(c4.y); cpv[4 * g + 2] = from_bits<V>(c4.z);
+        cpv[4 * g + 3] = from_bits<V>(c4.w);
     }
     const V corner = sm.corner[q];
     if (!Cfg::WPUB && lane == 31 && J > 0) {
         uint64_t* rs = p.row_slots + tidx * TR + row0;
 #pragma unroll
         for (int r = 0; r < RPW; r += 2)
-            st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][3] + rt[r])),
-                          pack(epoch, kIncl, to_bits(v[r + 1][3] + rt[r + 1])), pol);
+            st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][X - 1] + rt[r])),
+                          pack(epoch, kIncl, to_bits(v[r + 1][X - 1] + rt[r + 1])), pol);
     }
     if (!Cfg::WPUB && warp == NW - 1) {
         if (I > 0) {
-            uint64_t* cs = p.col_slots + tidx * TC + col0;
-            st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + cpv[0])),
-                          pack(epoch, kIncl, to_bits(v[RPW - 1][1] + cpv[1])), pol);
-            st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(v[RPW - 1][2] + cpv[2])),
-                          pack(epoch, kIncl, to_bits(v[RPW - 1][3] + cpv[3])), pol);
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                uint64_t* cs = p.col_slots + tidx * TC + g * 128 + col0;
+                const V* b = &v[RPW - 1][4 * g];
+                const V* c = &cpv[4 * g];
+                st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(b[0] + c[0])), pack(epoch, kIncl, to_bits(b[1] + c[1])),
+                              pol);
+                st_relaxed2_p(cs + 2, pack(epoch, kIncl, to_bits(b[2] + c[2])),
+                              pack(epoch, kIncl, to_bits(b[3] + c[3])), pol);
+            }
         }
         if (lane == 31) {  // GLS = total + rp[TR-1] + cp[TC-1];  GS = GS(I-1,J-1) + GLS
-            const V gls = v[RPW - 1][3] + rt[RPW - 1] + cpv[3];
+            const V gls = v[RPW - 1][X - 1] + rt[RPW - 1] + cpv[X - 1];
             st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(corner + gls)), pol);
         }
     }
-    V colterm[4];
+    V colterm[X];
 #pragma unroll
-    for (int c = 0; c < 4; ++c) colterm[c] = cpv[c] + corner;
+    for (int x = 0; x < X; ++x) colterm[x] = cpv[x] + corner;
     if constexpr (CARRY) {
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            const long long gj = static_cast<long long>(J) * TC + col0 + c;
-            colterm[c] = colterm[c] + (gj < p.cols ? p.carry[gj] : V(0));
+        for (int x = 0; x < X; ++x) {
+            const long long gj = static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4);
+            colterm[x] = colterm[x] + (gj < p.cols ? p.carry[gj] : V(0));
         }
     }
 #pragma unroll
     for (int r = 0; r < RPW; ++r)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + (rt[r] + colterm[c]);
+        for (int x = 0; x < X; ++x) v[r][x] = v[r][x] + (rt[r] + colterm[x]);
     const bool ragged = !TMA || ((J == p.C - 1) && (p.cols & 3) != 0);
     if (Cfg::DIRECT && !ragged) {
         // Step 4 store straight from registers: a lane writes 16 contiguous bytes of each of its rows
@@ -431,8 +528,11 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
         if (warp == 0 && lane == 0) WS_ST(kWsFastHits, o1 - o0);
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
-            *reinterpret_cast<uint4*>(&sm.out[(row0 + r) * TC + col0]) =
-                make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3]));
+#pragma unroll
+            for (int g = 0; g < G; ++g)
+                *reinterpret_cast<uint4*>(&sm.out[tm_sidx<Cfg>(row0 + r, g * 128 + col0)]) =
+                    make_uint4(to_bits(v[r][4 * g]), to_bits(v[r][4 * g + 1]), to_bits(v[r][4 * g + 2]),
+                               to_bits(v[r][4 * g + 3]));
         fence_proxy_async_smem();
         if constexpr (Cfg::QS) {
             __syncwarp();
@@ -443,9 +543,9 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
         for (int r = 0; r < RPW; ++r) {
             const long long gi = static_cast<long long>(I) * TR + row0 + r;
 #pragma unroll
-            for (int c = 0; c < 4; ++c) {
-                const long long gj = static_cast<long long>(J) * TC + col0 + c;
-                if (gi < p.rows && gj < p.cols) p.dst[gi * p.pitch + gj] = v[r][c];
+            for (int x = 0; x < X; ++x) {
+                const long long gj = static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4);
+                if (gi < p.rows && gj < p.cols) p.dst[gi * p.pitch + gj] = v[r][x];
             }
         }
     }
@@ -721,7 +821,10 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 WS_ST(kWsStResultWait, u1 - u0);
                 const bool ragged = !TMA || ((ti.J == p.C - 1) && (p.cols & 3) != 0);
                 if (!Cfg::DIRECT && !Cfg::QS && !ragged) {
-                    tma_store_2d_hint(&map_out, sm.out, ti.J * TC, ti.I * TR, spol);
+#pragma unroll
+                    for (int bx = 0; bx < Cfg::NB; ++bx)
+                        tma_store_2d_hint(&map_out, sm.out + bx * TR * Cfg::TB, ti.J * TC + bx * Cfg::TB, ti.I * TR,
+                                          spol);
                     bulk_commit();
 #if SAT_STATS
                     if (p.trace) p.trace[8LL * ti.t + 6] = static_cast<long long>(globaltimer_ns());
@@ -767,7 +870,10 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 if (TMA && valid) {
                     WS_ST(kWsLdIssue, 1);
                     mbar_arrive_expect_tx(&sm.full[sl.s], kTileBytes);
-                    tma_load_2d(sm.stage[sl.s], &map_in, &sm.full[sl.s], ti.J * TC, ti.I * TR, policy);
+#pragma unroll
+                    for (int bx = 0; bx < Cfg::NB; ++bx)
+                        tma_load_2d(sm.stage[sl.s] + bx * TR * Cfg::TB, &map_in, &sm.full[sl.s],
+                                    ti.J * TC + bx * Cfg::TB, ti.I * TR, policy);
 #if SAT_STATS
                     if (p.trace) p.trace[8LL * ti.t + 7] = static_cast<long long>(globaltimer_ns());
 #endif

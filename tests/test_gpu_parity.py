@@ -105,7 +105,7 @@ def test_int32_bit_exact(sat, shape):
     assert_i32_exact(run_sat(sat, a), a)
 
 
-@pytest.mark.parametrize("variant", range(12))
+@pytest.mark.parametrize("variant", range(16))
 @pytest.mark.parametrize("order", [0, 1])
 def test_int32_every_variant_and_order(sat, variant, order):
     if variant >= sat.num_variants():
@@ -119,7 +119,7 @@ def test_int32_every_variant_and_order(sat, variant, order):
             pytest.skip(str(e))
         raise
     try:
-        for shape in [(1000, 1000), (257, 3000), (4096, 130)]:
+        for shape in [(1000, 1000), (257, 3000), (4096, 130), (100, 2050)]:
             a = satgen.gen_host(*shape, seed=99 + variant, dist="u32")
             assert_i32_exact(run_sat(sat, a), a)
     finally:
@@ -455,7 +455,9 @@ def test_sharded_nccl_single_rank():
 # ----------------------------------------------------------------------------- queries on a SAT
 @pytest.mark.parametrize("shape,pitch,rh,rw", [((1, 1), None, 0, 0), ((300, 517), None, 3, 5), ((129, 257), 264, 0, 7),
                                                ((64, 1000), None, 40, 1), ((1009, 203), 208, 12, 12),
-                                               ((50, 60), None, 100, 100)])
+                                               ((50, 60), None, 100, 100), ((300, 516), None, 3, 5),
+                                               ((40, 3001), 3004, 2, 700), ((33, 2500), None, 1, 1500),
+                                               ((20, 5000), None, 25, 0), ((7, 4), None, 0, 3)])
 def test_box_sum_int32_bit_exact(sat, shape, pitch, rh, rw):
     b = satgen.gen_host(*shape, seed=31 + shape[0], dist="u32")  # any matrix is a valid operand of P:48
     buf, bd = dev_copy(b, pitch)
@@ -470,7 +472,8 @@ def test_box_sum_int32_bit_exact(sat, shape, pitch, rh, rw):
         assert (full[:, shape[1]:] == 0x5A5A5A5A).all(), "pad elements were written"
 
 
-@pytest.mark.parametrize("shape,rh,rw", [((333, 444), 4, 9), ((128, 128), 0, 0), ((1, 2049), 0, 30)])
+@pytest.mark.parametrize("shape,rh,rw", [((333, 444), 4, 9), ((128, 128), 0, 0), ((1, 2049), 0, 30),
+                                         ((65, 2052), 7, 300)])
 def test_box_sum_fp32_bit_exact(sat, shape, rh, rw):
     b = satgen.gen_host(*shape, seed=77, dist="fsym")
     _, bd = dev_copy(b)
