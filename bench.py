@@ -136,6 +136,14 @@ def cpu_oracle_sample(rows: int, cols: int, dtype: str, target_s: float = 12.0) 
 
 
 # ------------------------------------------------------------------------------------- helpers
+def order_name(order: int) -> str:
+    """Tile order of the plan: 0 anti-diagonal (Fig. 9), 1 row-major, (g << 8) diagonal of g-tile groups."""
+    g = (order >> 8) & 255
+    if (order & 15) == 0 and g > 1:
+        return f"anti-diagonal of {g}-tile groups"
+    return ["anti-diagonal", "row-major"][order & 15]
+
+
 def load_ncu_traffic(workload: str):
     p = ROOT / "profiles" / "ncu_summary.json"
     if not p.exists():
@@ -336,7 +344,7 @@ def main():
             "data": "synthetic (seeded splitmix64 counter generator, uniform; generated in HBM)",
             "config": {"workload": workload, "rows": rows, "cols": cols, "pitch": cols,
                        "tile": [plan["tile_rows"], plan["tile_cols"]], "ctas": plan["ctas"],
-                       "variant": plan["variant"], "order": ["diagonal", "row-major"][plan["order"]],
+                       "variant": plan["variant"], "order": order_name(plan["order"]),
                        "l2": "inputs (4 B x n^2) larger than the 126 MB L2; no flush",
                        "parallelism": "single GPU" if world == 1 else f"strips x{world}"},
             "hbm_gbs": achieved,

@@ -98,9 +98,9 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
 };
 
-template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC>
-struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC>> {
-    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC>;
+template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC, int LB>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB>;
     static constexpr int box_cols = Cfg::TB;
     static constexpr int out_box_rows = Cfg::OBR;
     static constexpr int threads = Cfg::THREADS;
@@ -222,9 +222,13 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 8
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),  // 9
         make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>>(),  // 10: u8 integral images only (4 stages of 16 KiB u8 tiles)
-        make_variant<sat::TmCfg<8, 2, 5, 1, 3, 4, 0, 0, 32, 512>>(),   // 11: flat 32 x 512 tiles, 8 compute warps
-        make_variant<sat::TmCfg<16, 2, 5, 1, 3, 4, 0, 0, 64, 256>>(),  // 12: flat 64 x 256 tiles
-        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),   // 13: flat 64 x 256 tiles, 8 compute warps
+        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),    // 11: flat 64 x 256 tiles, 8 compute warps, ring of 8
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 64, 256>>(),    // 12: ... ring of 7
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 13: ... ring of 6
+        make_variant<sat::TmCfg<8, 2, 10, 1, 3, 4, 0, 0, 64, 256>>(),   // 14: ... ring of 10
+        make_variant<sat::TmCfg<16, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),   // 15: 16 compute warps, ring of 8
+        make_variant<sat::TmCfg<8, 2, 12, 1, 3, 4, 0, 0, 64, 256>>(),   // 16: ring of 12
+        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 32, 512>>(),    // 17: flat 32 x 512 tiles, ring of 8
     };
     return vs;
 }
@@ -239,8 +243,17 @@ int g_max_ctas = 0;
 int auto_variant(int64_t rows, int64_t cols) {
     // measured device times (tools/graph_sweep.py, tools/sweep_variants.py): up to
     // ~1.4K x 1.4K (<= 128 tiles of 128^2) the classic kernel with 64 x 128 tiles has the shortest
-    // latency; above, the TMEM-parked kernel with decoupled walkers (parking depth 4)
-    return rows * cols <= (int64_t(1) << 21) ? 4 : 9;
+    // latency; above, the TMEM-parked kernel with decoupled walkers (parking depth 4) on flat
+    // 64 x 256 tiles
+    const int64_t n = rows * cols;
+    return n <= (int64_t(1) << 21) ? 4 : (n <= (int64_t(1) << 25) ? 9 : 13);
+}
+
+int auto_order(int vi, int64_t cols) {
+    // flat 64 x 256 tiles with >= 128 tile columns (>= 32K columns): anti-diagonal order of 2-wide tile
+    // groups (each DRAM row visit 2 KiB); narrower grids keep the plain anti-diagonal order, which
+    // measured faster there (tools/sweep_variants.py, profiles/r01_sweep_sizes.jsonl)
+    return (vi == 13 && (cols + 255) / 256 >= 128) ? 0x200 : 0;
 }
 
 // ------------------------------------------------------------------ device info caches
@@ -451,7 +464,7 @@ sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* sr
     {
         std::lock_guard<std::mutex> lk(g_mu);
         vi = g_variant >= 0 ? g_variant : (u8 ? 10 : auto_variant(rows, cols));
-        order = g_order;
+        order = (g_variant < 0 && g_order == 0) ? auto_order(vi, cols) : g_order;
     }
     const Variant& v = variants()[vi];
     pl->vi = vi;
@@ -664,9 +677,9 @@ sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, in
     if (gy > 65535) gy = 65535;
     const dim3 grid(static_cast<unsigned>(gx), static_cast<unsigned>(gy));
     const bool vec = ((reinterpret_cast<uintptr_t>(out) & 15u) == 0) && ((pitch * 4) % 16 == 0);
-    // staged kernel: both pointers 16-byte aligned and the two double-buffered row segments in 48 KB
+    // staged kernel: both pointers 16-byte aligned and kBoxBufs pairs of row segments in 48 KB
     const int64_t nv = (sat::kBoxPanel + 2 * rw + 8) / 4 + 1;
-    const size_t smem = static_cast<size_t>(nv) * 4 * 4 * 4;
+    const size_t smem = static_cast<size_t>(nv) * 4 * 4 * 2 * sat::kBoxBufs;
     if (vec && ((reinterpret_cast<uintptr_t>(b) & 15u) == 0) && smem <= 48 * 1024) {
         if (dt == SAT_INT32)
             sat::box_sum_smem_kernel<uint32_t><<<grid, sat::kBoxThreads, smem, st>>>(
@@ -1017,9 +1030,9 @@ SAT_API sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm) {
     if (variant < -1 || variant >= static_cast<int>(variants().size()))
         return fail(SAT_ERR_INVALID_VALUE, "unknown variant %d", variant);
 #if SAT_STATS
-    if (order < 0 || (order & 15) > 1) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
+    if (order < 0 || (order & 15) > 1 || order > 0xffff) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
 #else
-    if (order < 0 || order > 1) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
+    if (order < 0 || (order & ~0xff01) != 0) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
 #endif
     if (ctas_per_sm < 0) return fail(SAT_ERR_INVALID_VALUE, "ctas_per_sm < 0");
     std::lock_guard<std::mutex> lk(g_mu);
@@ -1047,7 +1060,7 @@ SAT_API sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* 
 }
 
 SAT_API sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out, void* stream) {
-    if (R <= 0 || C <= 0 || R * C > (int64_t(1) << 30) || !out || order < 0 || order > 1)
+    if (R <= 0 || C <= 0 || R * C > (int64_t(1) << 30) || !out || order < 0 || (order & ~0xff01) != 0)
         return fail(SAT_ERR_INVALID_VALUE, "bad args");
     const int64_t n = R * C;
     int blocks = static_cast<int>((n + 255) / 256);

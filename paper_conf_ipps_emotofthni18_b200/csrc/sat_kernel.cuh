@@ -100,13 +100,7 @@ __device__ __forceinline__ long long tri_floor_inv(long long s) {  // largest k 
     return k;
 }
 
-__device__ __forceinline__ void tile_of_serial(int s_, int R, int C, int order, int& I, int& J) {
-    if ((order & 15) == 1) {
-        I = s_ / C;
-        J = s_ - I * C;
-        return;
-    }
-    const long long s = s_;
+__device__ __forceinline__ void diag_of_serial(long long s, int R, int C, int& I, int& J) {
     const long long m = R < C ? R : C, M = R < C ? C : R;
     const long long headA = tri(m);            // tiles on diagonals d < m
     const long long headB = headA + (M - m) * m;  // ... on diagonals d < M
@@ -126,6 +120,27 @@ __device__ __forceinline__ void tile_of_serial(int s_, int R, int C, int order, 
     const long long i0 = d - C + 1 > 0 ? d - C + 1 : 0;
     I = static_cast<int>(i0 + (s - base));
     J = static_cast<int>(d - I);
+}
+
+// order & 15: 0 = anti-diagonal (Fig. 9), 1 = row-major.  (order >> 8) & 255 = g > 1 with order & 15
+// == 0 and g | C: anti-diagonal order of g-wide tile groups, the g tiles of a group consecutive and
+// left to right (a topological order too: a tile's left neighbour is earlier in its group or on the
+// previous group diagonal, its upper neighbours on the previous group diagonal).  The g tiles of a
+// group share their DRAM rows, so the rows concurrent tiles touch are g times longer.
+__device__ __forceinline__ void tile_of_serial(int s_, int R, int C, int order, int& I, int& J) {
+    if ((order & 15) == 1) {
+        I = s_ / C;
+        J = s_ - I * C;
+        return;
+    }
+    const int g = (order >> 8) & 255;
+    if (g > 1 && C % g == 0) {
+        int J2;
+        diag_of_serial(s_ / g, R, C / g, I, J2);
+        J = J2 * g + s_ % g;
+        return;
+    }
+    diag_of_serial(s_, R, C, I, J);
 }
 
 // ------------------------------------------------------------------ look-backs

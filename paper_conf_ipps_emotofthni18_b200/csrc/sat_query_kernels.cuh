@@ -68,26 +68,29 @@ __global__ void __launch_bounds__(256) box_sum_kernel(const V* __restrict__ b, V
 // the same left-to-right order as box_sum_kernel.  Global traffic per
 // output row: one read of each SAT row segment (row u is row d of the output row 2*rh+1 above, an L2
 // hit) and coalesced streaming stores, instead of 16 scalar L2 loads per 4 outputs.
-// Requires pitch * 4 and both pointers 16-byte aligned (VEC).  Double-buffered: the segments of the
-// next row are loaded while the current row is evaluated.
+// Requires pitch * 4 and both pointers 16-byte aligned (VEC).  The segments of the next kBoxBufs - 1
+// rows are in flight (cp.async) while the current row is evaluated.
 constexpr int kBoxThreads = 256;
 constexpr int kBoxPanel = 4 * kBoxThreads;
+
+constexpr int kBoxBufs = 3;  // row-segment pairs in flight per block (cp.async groups)
 
 template <typename V>
 __device__ __forceinline__ void box_load_seg(const V* __restrict__ b, int64_t pitch, int64_t row, int64_t a0,
                                              int64_t hi, int nv, V* seg) {
-    // seg[k] = b[row][a0 + k] for a0 + k in [0, hi], else 0 (a0 is a multiple of 4; hi = last column)
+    // seg[k] = b[row][a0 + k] for a0 + k in [0, hi], else 0 (a0 is a multiple of 4; hi = last column);
+    // 16-byte cp.async with a source size of 0..16 bytes (the rest of the 16 bytes is zero-filled)
     for (int q = threadIdx.x; q < nv; q += blockDim.x) {
         const int64_t j = a0 + 4 * static_cast<int64_t>(q);
-        uint4 w = make_uint4(0u, 0u, 0u, 0u);
-        if (row >= 0 && j >= 0 && j <= hi) w = __ldcg(reinterpret_cast<const uint4*>(b + row * pitch + j));
-        if (row >= 0 && j + 3 > hi) {  // columns past the last one read as zero (within the pitch row)
-            if (j + 1 > hi) w.y = 0u;
-            if (j + 2 > hi) w.z = 0u;
-            if (j + 3 > hi) w.w = 0u;
-            if (j > hi) w.x = 0u;
+        int bytes = 0;
+        const V* src = b;
+        if (row >= 0 && j >= 0 && j <= hi) {
+            bytes = (hi - j + 1 >= 4) ? 16 : static_cast<int>(hi - j + 1) * 4;
+            src = b + row * pitch + j;
         }
-        *reinterpret_cast<uint4*>(seg + 4 * q) = w;
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_addr(seg + 4 * q)), "l"(src),
+                     "r"(bytes)
+                     : "memory");
     }
 }
 
@@ -96,23 +99,30 @@ __global__ void __launch_bounds__(kBoxThreads) box_sum_smem_kernel(const V* __re
                                                                    int64_t rows, int64_t cols, int64_t pitch,
                                                                    int64_t rh, int64_t rw, int nv) {
     extern __shared__ __align__(16) unsigned char box_smem[];
-    V* buf = reinterpret_cast<V*>(box_smem);  // [2 buffers][2 rows (d, u)][4 * nv]
+    V* buf = reinterpret_cast<V*>(box_smem);  // [kBoxBufs][2 rows (d, u)][4 * nv]
     const int64_t p0 = static_cast<int64_t>(blockIdx.x) * kBoxPanel;
     const int64_t a0 = ((p0 - rw - 1) >= 0) ? ((p0 - rw - 1) & ~int64_t(3)) : -((-(p0 - rw - 1) + 3) & ~int64_t(3));
     const int64_t hi = cols - 1;
     const int seglen = 4 * nv;
-    auto load_row = [&](int64_t i, int sb) {
-        const int64_t u = i - rh - 1;
-        const int64_t d = i + rh < rows - 1 ? i + rh : rows - 1;
-        box_load_seg(b, pitch, d, a0, hi, nv, buf + (2 * sb) * seglen);
-        box_load_seg(b, pitch, u, a0, hi, nv, buf + (2 * sb + 1) * seglen);
+    auto load_row = [&](int64_t i, int sb) {  // always commits one group (empty past the last row)
+        if (i < rows) {
+            const int64_t u = i - rh - 1;
+            const int64_t d = i + rh < rows - 1 ? i + rh : rows - 1;
+            box_load_seg(b, pitch, d, a0, hi, nv, buf + (2 * sb) * seglen);
+            box_load_seg(b, pitch, u, a0, hi, nv, buf + (2 * sb + 1) * seglen);
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
     };
-    int sb = 0;
+    const int64_t step = gridDim.y;
     int64_t i = blockIdx.y;
-    if (i < rows) load_row(i, 0);
-    for (; i < rows; i += gridDim.y) {
-        __syncthreads();  // segments of row i are in buffer sb; buffer sb^1 is free
-        if (i + gridDim.y < rows) load_row(i + gridDim.y, sb ^ 1);
+#pragma unroll
+    for (int k = 0; k < kBoxBufs - 1; ++k) load_row(i + k * step, k);
+    int sb = 0;
+    for (; i < rows; i += step) {
+        asm volatile("cp.async.wait_group %0;" ::"n"(kBoxBufs - 2) : "memory");
+        __syncthreads();  // row i's segments are visible to the block; every thread is done with row i - step
+        // prefetch row i + (kBoxBufs-1) step into the buffer of row i - step
+        load_row(i + (kBoxBufs - 1) * step, (sb + kBoxBufs - 1) % kBoxBufs);
         const V* D = buf + (2 * sb) * seglen;
         const V* U = D + seglen;
         V* dst = out + i * pitch;
@@ -126,8 +136,9 @@ __global__ void __launch_bounds__(kBoxThreads) box_sum_smem_kernel(const V* __re
                 __stcs(dst + j, ((D[kr] - U[kr]) - D[kl]) + U[kl]);
             }
         }
-        sb ^= 1;
+        sb = (sb + 1) % kBoxBufs;
     }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
 
 // Batched rectangle queries: rects[k] = (u, d, l, r) in the convention of P:48 (u < i <= d,

@@ -29,8 +29,9 @@ namespace sat {
 // TR_ x TC_ tiles: TC_ = 128 * G (a lane owns G chunks of 4 columns, 128 apart); flat tiles (TC_ > 128)
 // keep the tile's 64 KiB but make every DRAM row visit 4 B * TC_ long (tile shape).
 template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0, int QS_ = 0,
-          int TR_ = 128, int TC_ = 128>
+          int TR_ = 128, int TC_ = 128, int LB_ = 2>
 struct TmCfg {
+    static constexpr int LB = LB_;                  // row / column look-back: predecessors polled per round
     static constexpr int TR = TR_, TC = TC_, NW = NW_;
     static constexpr int G = TC / 128;             // column chunks per lane
     static constexpr int TB = TC < 256 ? TC : 256;  // TMA box width (boxDim <= 256 elements)
@@ -270,22 +271,54 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
     for (int r = 1; r < RPW; ++r)
 #pragma unroll
         for (int x = 0; x < X; ++x) v[r][x] = v[r][x] + v[r - 1][x];
+    if constexpr (G == 1) {
 #pragma unroll
-    for (int r = 0; r < RPW; ++r) {
-        V carry = V(0);  // row total of the chunks to the left
-#pragma unroll
-        for (int g = 0; g < G; ++g) {
-            V* w = &v[r][4 * g];
+        for (int r = 0; r < RPW; ++r) {
+            V* w = &v[r][0];
             w[1] = w[1] + w[0];
             w[2] = w[2] + w[1];
             w[3] = w[3] + w[2];
             const V incl = warp_inclusive_scan(w[3], lane);
             V excl = __shfl_up_sync(kFull, incl, 1);
             if (lane == 0) excl = V(0);
-            if (g > 0) excl = excl + carry;
 #pragma unroll
             for (int c = 0; c < 4; ++c) w[c] = w[c] + excl;
-            if (g + 1 < G) carry = carry + __shfl_sync(kFull, incl, 31);
+        }
+    } else {
+        // RPW x G independent warp scans, step-major so that their shuffles overlap
+        V incl[RPW][G];
+#pragma unroll
+        for (int r = 0; r < RPW; ++r)
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                V* w = &v[r][4 * g];
+                w[1] = w[1] + w[0];
+                w[2] = w[2] + w[1];
+                w[3] = w[3] + w[2];
+                incl[r][g] = w[3];
+            }
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1)
+#pragma unroll
+            for (int r = 0; r < RPW; ++r)
+#pragma unroll
+                for (int g = 0; g < G; ++g) {
+                    const V y = __shfl_up_sync(kFull, incl[r][g], d);
+                    if (lane >= d) incl[r][g] = incl[r][g] + y;
+                }
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            V carry = V(0);  // row total of the chunks to the left
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                V excl = __shfl_up_sync(kFull, incl[r][g], 1);
+                if (lane == 0) excl = V(0);
+                if (g > 0) excl = excl + carry;
+                V* w = &v[r][4 * g];
+#pragma unroll
+                for (int c = 0; c < 4; ++c) w[c] = w[c] + excl;
+                if (g + 1 < G) carry = carry + __shfl_sync(kFull, incl[r][g], 31);
+            }
         }
     }
     {   // band offsets: warp w adds the bottoms of bands 0 .. w-1 (no serial scan)
@@ -558,6 +591,33 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
     if (warp == 0 && lane == 0) WS_ST(kWsFinish, c2 - c1);
 }
 
+// Look-back step over up to NP predecessors loaded in one round (w[h] = words of predecessor pos - h):
+// consumed in order until one has a not-yet-published element that is still pending.
+template <typename V, int E, int NP>
+__device__ __forceinline__ bool lb_consume_n(uint32_t& pending, int& pos, V (&acc)[E], const uint64_t (&w)[NP][E],
+                                             uint32_t epoch) {
+    bool progress = false;
+#pragma unroll
+    for (int h = 0; h < NP; ++h) {
+        if (!pending || pos < 0) break;
+        bool ok = true;
+#pragma unroll
+        for (int e = 0; e < E; ++e)
+            if (((pending >> e) & 1u) && !word_ready(w[h][e], epoch)) ok = false;
+        if (!ok) break;
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+            if ((pending >> e) & 1u) {
+                acc[e] = acc[e] + from_bits<V>(static_cast<uint32_t>(w[h][e]));
+                if (word_kind(w[h][e]) == kIncl) pending &= ~(1u << e);
+            }
+        }
+        pos -= 1;
+        progress = true;
+    }
+    return progress;
+}
+
 // Walker with a decoupled diagonal look-back (Cfg::DECOUPLED), one tile at a time, in acquisition order.
 //
 // Row walker: row look-back (Step 2.A.2) and diagonal look-back (Step 3.2).  Column
@@ -582,6 +642,8 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
     constexpr int TR = Cfg::TR, TC = Cfg::TC, RPW = Cfg::RPW, NW = Cfg::NW;
     constexpr int E = ROW ? Cfg::ER : Cfg::EC;
     constexpr int DW = 4;  // diagonal predecessors polled per round
+    // predecessors polled per round: LB, capped at 32 words (64 registers) per lane
+    constexpr int NP = Cfg::LB * E <= 32 ? Cfg::LB : (32 / E >= 1 ? 32 / E : 1);
     const uint64_t pol = policy_evict_last();
     auto flag = [&](const int* f) { return *reinterpret_cast<const volatile int*>(f); };
     for (Slot<Cfg::NQ> nx;; nx.next()) {
@@ -606,20 +668,20 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
         bool cin = false, lpub = false;
         while (true) {
             // ---- issue this round's loads
-            uint64_t w0[E], w1[E], wd = 0;
-            const bool have1 = pos >= 1;
+            uint64_t w[NP][E], wd = 0;
             if (pend) {
                 const uint64_t* q = own - (ROW ? static_cast<long long>(J - pos) * TR
                                                : static_cast<long long>(I - pos) * p.C * TC) + lane * E;
-                ld_words_p<E>(q, w0, pol);
-                if (have1) ld_words_p<E>(q - step, w1, pol);
+#pragma unroll
+                for (int h = 0; h < NP; ++h)
+                    if (pos - h >= 0) ld_words_p<E>(q - h * step, w[h], pol);
             }
             const int kk = dbase + lane;
             const bool dinr = ROW && !ddone && lane < DW && (I - kk >= 0) && (J - kk >= 0);
             if (dinr) wd = ld_relaxed_p(p.corner_slots + static_cast<long long>(I - kk) * p.C + (J - kk), pol);
             // ---- consume
             bool progress = false;
-            if (pend) progress = lb_consume<V, E>(pend, pos, acc, w0, w1, have1, epoch);
+            if (pend) progress = lb_consume_n<V, E, NP>(pend, pos, acc, w, epoch);
             if (ROW && !ddone) {
                 const bool ready = !dinr || word_ready(wd, epoch);
                 const unsigned incl = __ballot_sync(kFull, dinr && ready && word_kind(wd) == kIncl);

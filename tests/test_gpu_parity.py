@@ -105,8 +105,8 @@ def test_int32_bit_exact(sat, shape):
     assert_i32_exact(run_sat(sat, a), a)
 
 
-@pytest.mark.parametrize("variant", range(16))
-@pytest.mark.parametrize("order", [0, 1])
+@pytest.mark.parametrize("variant", range(20))
+@pytest.mark.parametrize("order", [0, 1, 0x400])
 def test_int32_every_variant_and_order(sat, variant, order):
     if variant >= sat.num_variants():
         pytest.skip("no such variant")
@@ -349,6 +349,24 @@ def test_device_tile_order_matches_fig9_order(sat, R, C):
     assert (got == want).all()
     rm = sat.debug_tile_order(R, C, 1).cpu().numpy()
     assert (rm == np.array([(I, J) for I in range(R) for J in range(C)])).all()
+
+
+@pytest.mark.parametrize("R,C,g", [(5, 8, 2), (64, 128, 4), (512, 128, 8), (3, 12, 4), (7, 9, 3), (6, 10, 4)])
+def test_device_grouped_tile_order_is_topological(sat, R, C, g):
+    """Anti-diagonal order of g-wide groups: a permutation of the R x C tiles in which every tile's left,
+    upper and upper-left neighbours come first (the look-back's dependencies); with
+    g not dividing C the plain Fig. 9 order is used."""
+    got = sat.debug_tile_order(R, C, g << 8).cpu().numpy()
+    if C % g:
+        assert (got == np.array(oracle.tile_order(R, C))).all()
+        return
+    assert sorted(map(tuple, got.tolist())) == [(I, J) for I in range(R) for J in range(C)]
+    pos = {tuple(t): k for k, t in enumerate(got.tolist())}
+    for (I, J), k in pos.items():
+        for dep in [(I, J - 1), (I - 1, J), (I - 1, J - 1)]:
+            if dep[0] >= 0 and dep[1] >= 0:
+                assert pos[dep] < k
+    assert [tuple(t) for t in got[:g].tolist()] == [(0, j) for j in range(g)]
 
 
 # ----------------------------------------------------------------------------------- full-size (BASELINE configs)
