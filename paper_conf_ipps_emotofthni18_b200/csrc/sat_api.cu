@@ -226,9 +226,6 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 64, 256>>(),    // 12: ... ring of 7
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 13: ... ring of 6
         make_variant<sat::TmCfg<8, 2, 10, 1, 3, 4, 0, 0, 64, 256>>(),   // 14: ... ring of 10
-        make_variant<sat::TmCfg<16, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),   // 15: 16 compute warps, ring of 8
-        make_variant<sat::TmCfg<8, 2, 12, 1, 3, 4, 0, 0, 64, 256>>(),   // 16: ring of 12
-        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 32, 512>>(),    // 17: flat 32 x 512 tiles, ring of 8
     };
     return vs;
 }

@@ -36,7 +36,7 @@ struct TmCfg {
     static constexpr int G = TC / 128;             // column chunks per lane
     static constexpr int TB = TC < 256 ? TC : 256;  // TMA box width (boxDim <= 256 elements)
     static constexpr int NB = TC / TB;              // TMA boxes per tile (stage / output layout [NB][TR][TB])
-    static constexpr bool SBAND = TC > 128;         // band bottoms exchanged through the tile's input stage
+    static constexpr bool SBAND = TC > 128;         // single-parity band buffer (two barriers per tile)
     static constexpr int IN = IN_;    // input stages
     static constexpr int STAGES = IN;
     static constexpr int NQ = NQ_;    // tile ring
@@ -59,7 +59,7 @@ struct TmCfg {
     static_assert(NW % 4 == 0 && TR % NW == 0 && RPW % 4 == 0, "compute warps cover the 4 TMEM lane quarters");
     static_assert(NREG == 16 || NREG == 32 || NREG == 64, "tcgen05 32x32b.x16 / .x32 parking");
     static_assert(TC % 128 == 0 && TC % TB == 0 && TR >= 32 && TR * TC == 128 * 128, "64 KiB tiles, TC = 128 G");
-    static_assert(!SBAND || (NW <= TR && !DIRECT && !QS), "flat tiles: band rows fit in a stage, TMA stores");
+    static_assert(!SBAND || (!DIRECT && !QS), "flat tiles: TMA stores");
     static_assert(D >= 2 && D * TM_COLS_PER_SLOT <= 512, "TMEM columns");
     static_assert(IN >= 1 && NQ >= IN + D - 1 && NQ <= 16, "rings");
 };
@@ -68,7 +68,7 @@ template <typename V, typename Cfg, typename TIn = V>
 struct TmSmem {
     alignas(1024) TIn stage[Cfg::IN][Cfg::TR * Cfg::TC];  // input ring (TMA loads; u8 for integral images)
     alignas(1024) V out[Cfg::DIRECT ? 4 : Cfg::TR * Cfg::TC];  // GSAT of one tile (TMA store source)
-    alignas(16) V band[Cfg::SBAND ? 1 : 2][Cfg::SBAND ? 1 : Cfg::NW][Cfg::SBAND ? 4 : Cfg::TC];
+    alignas(16) V band[Cfg::SBAND ? 1 : 2][Cfg::NW][Cfg::TC];
     alignas(16) V rp[Cfg::NQ][Cfg::TR];
     alignas(16) V cp[Cfg::NQ][Cfg::TC];
     V corner[Cfg::NQ];
@@ -246,12 +246,9 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
             }
         }
     }
-    // the pixels are in registers: the loader may refill the stage now (flat tiles: after the band
-    // exchange, which goes through this stage)
-    if constexpr (!Cfg::SBAND) {
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.empty[s]);
-    }
+    // the pixels are in registers: the loader may refill the stage now
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sm.empty[s]);
     if (TMA && J == p.C - 1) {  // right edge: zero columns >= cols (16-byte TMA granules, reading R2)
 #pragma unroll
         for (int x = 0; x < X; ++x)
@@ -326,8 +323,8 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
 #pragma unroll
         for (int x = 0; x < X; ++x) off[x] = V(0);
         if constexpr (Cfg::SBAND) {
-            // every warp has read its rows of the stage: the stage holds the band bottoms (row w at w * TC)
-            V* bands = reinterpret_cast<V*>(sm.stage[s]);
+            // one band buffer: every warp is done with the previous tile's bottoms before it is rewritten
+            V* bands = &sm.band[0][0][0];
             named_bar_sync(1, NW * 32);
 #pragma unroll
             for (int g = 0; g < G; ++g)
@@ -344,10 +341,6 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
                     off[4 * g + 2] = off[4 * g + 2] + from_bits<V>(q.z);
                     off[4 * g + 3] = off[4 * g + 3] + from_bits<V>(q.w);
                 }
-            // generic-proxy writes to the stage precede the next TMA (async-proxy) write into it
-            fence_proxy_async_smem();
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&sm.empty[s]);
         } else {
             *reinterpret_cast<uint4*>(&sm.band[par][warp][col0]) = make_uint4(
                 to_bits(v[RPW - 1][0]), to_bits(v[RPW - 1][1]), to_bits(v[RPW - 1][2]), to_bits(v[RPW - 1][3]));
@@ -439,10 +432,6 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
             }
         }
     }
-    } else if constexpr (Cfg::SBAND) {
-        named_bar_sync(1, NW * 32);  // timing experiment: the stage may be refilled once every warp has read it
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&sm.empty[s]);
     }
     // park the block
     uint32_t r32[Cfg::NREG];
