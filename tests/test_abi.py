@@ -53,13 +53,18 @@ def test_variants_and_tuning(sat):
     n = sat.num_variants()
     assert n >= 1
     shapes = [sat.variant_info(v) for v in range(n)]
-    assert all(tc == 128 and tr % 32 == 0 for tr, tc in shapes)
+    # tiles of 64 KiB or less, 128 columns per lane chunk (flat 64 x 256 tiles are the production shape)
+    assert all(tc % 128 == 0 and tr % 32 == 0 and tr * tc <= 128 * 128 for tr, tc in shapes)
+    assert (64, 256) in shapes and (128, 128) in shapes
     with pytest.raises(sat.SatError):
         sat.variant_info(n)
     with pytest.raises(sat.SatError):
         sat.set_tuning(n, 0, 0)
     with pytest.raises(sat.SatError):
         sat.set_tuning(-1, 2, 0)
+    with pytest.raises(sat.SatError):
+        sat.set_tuning(-1, 0x201 | 0x10000, 0)
+    sat.set_tuning(-1, 0x200, 0)  # anti-diagonal order of 2-tile groups
     sat.set_tuning(-1, 0, 0)
     sat.set_max_ctas(0)
 
