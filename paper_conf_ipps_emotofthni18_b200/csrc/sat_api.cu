@@ -603,7 +603,8 @@ sat_status_t colsum_impl(sat_dtype_t dt, const void* src, void* colsum, int64_t 
     if (s != SAT_OK) return s;
     const bool vec = ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) && (pitch % 4 == 0);
     const int64_t bx = (cols + (vec ? 1023 : 255)) / (vec ? 1024 : 256);
-    int64_t nseg = (static_cast<int64_t>(di->sms) * 8 + bx - 1) / bx;
+    // one full wave: at most 8 blocks of 256 threads per SM (a partial second wave doubles the time)
+    int64_t nseg = (static_cast<int64_t>(di->sms) * 8) / bx;
     const int64_t max_seg = (rows + 7) / 8;
     if (nseg > max_seg) nseg = max_seg;
     if (nseg > 65535) nseg = 65535;
