@@ -98,9 +98,9 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
 };
 
-template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC, int LB>
-struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB>> {
-    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB>;
+template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC, int LB, int CT>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT>;
     static constexpr int box_cols = Cfg::TB;
     static constexpr int out_box_rows = Cfg::OBR;
     static constexpr int threads = Cfg::THREADS;
@@ -226,6 +226,9 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 64, 256>>(),    // 12: ... ring of 7
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 13: ... ring of 6
         make_variant<sat::TmCfg<8, 2, 10, 1, 3, 4, 0, 0, 64, 256>>(),   // 14: ... ring of 10
+        make_variant<sat::TmCfg<16, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),   // 15: 16 compute warps (4 rows each)
+        make_variant<sat::TmCfg<8, 3, 7, 1, 3, 4, 1, 0, 64, 256>>(),    // 16: GSAT stored from registers, 3 stages
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 1>>(),  // 17: variant 13, lanes own 8 contiguous columns
     };
     return vs;
 }

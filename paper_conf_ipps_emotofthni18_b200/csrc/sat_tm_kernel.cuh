@@ -29,8 +29,9 @@ namespace sat {
 // TR_ x TC_ tiles: TC_ = 128 * G (a lane owns G chunks of 4 columns, 128 apart); flat tiles (TC_ > 128)
 // keep the tile's 64 KiB but make every DRAM row visit 4 B * TC_ long (tile shape).
 template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0, int QS_ = 0,
-          int TR_ = 128, int TC_ = 128, int LB_ = 2>
+          int TR_ = 128, int TC_ = 128, int LB_ = 2, int CT_ = 0>
 struct TmCfg {
+    static constexpr bool CT = CT_ != 0;            // a lane owns 4 G contiguous columns (one warp scan per row)
     static constexpr int LB = LB_;                  // row / column look-back: predecessors polled per round
     static constexpr int TR = TR_, TC = TC_, NW = NW_;
     static constexpr int G = TC / 128;             // column chunks per lane
@@ -59,7 +60,8 @@ struct TmCfg {
     static_assert(NW % 4 == 0 && TR % NW == 0 && RPW % 4 == 0, "compute warps cover the 4 TMEM lane quarters");
     static_assert(NREG == 16 || NREG == 32 || NREG == 64, "tcgen05 32x32b.x16 / .x32 parking");
     static_assert(TC % 128 == 0 && TC % TB == 0 && TR >= 32 && TR * TC == 128 * 128, "64 KiB tiles, TC = 128 G");
-    static_assert(!SBAND || (!DIRECT && !QS), "flat tiles: TMA stores");
+    static_assert(!SBAND || !QS, "flat tiles: whole-tile TMA stores");
+    static_assert(!CT || (TC == 256 && !DIRECT), "contiguous lane columns: 64 x 256 tiles");
     static_assert(D >= 2 && D * TM_COLS_PER_SLOT <= 512, "TMEM columns");
     static_assert(IN >= 1 && NQ >= IN + D - 1 && NQ <= 16, "rings");
 };
@@ -167,6 +169,12 @@ __device__ __forceinline__ uint32_t tm_addr(uint32_t base, int warp, int slot) {
            static_cast<uint32_t>(slot * Cfg::TM_COLS_PER_SLOT + (warp >> 2) * Cfg::NREG);
 }
 
+// First column (within the tile) of chunk g of a lane: chunks 128 apart, or 4 G contiguous columns (CT)
+template <typename Cfg>
+__device__ __forceinline__ int tm_cb(int lane, int g) {
+    return Cfg::CT ? lane * 4 * Cfg::G + 4 * g : g * 128 + lane * 4;
+}
+
 // Element (r, c) of a stage / the output buffer: NB boxes of TR x TB, each row-major.
 template <typename Cfg>
 __device__ __forceinline__ constexpr int tm_sidx(int r, int c) {
@@ -200,7 +208,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW, G = Cfg::G, X = 4 * Cfg::G;
     static_assert(sizeof(TIn) != 1 || TC == 128, "u8 tiles: 128 columns");
     const int s = sl.s;
-    const int row0 = warp * RPW, col0 = lane * 4;  // this lane's columns: g * 128 + col0 + c
+    const int row0 = warp * RPW, col0 = lane * 4;  // this lane's columns: tm_cb<Cfg>(lane, g) + c
     SAT_CLK(c0);
     mbar_wait(&sm.full[s], sl.ph);
     SAT_CLK(c1);
@@ -223,13 +231,26 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
 #pragma unroll
             for (int c = 0; c < 4; ++c) v[r][c] = V((w >> (8 * c)) & 0xffu);
         }
+    } else if constexpr (TMA && Cfg::CT) {
+        // two 16-byte halves per row, the lanes of each quarter-warp in swapped order (conflict-free)
+        const TIn* tile = sm.stage[s];
+        const int swz = (lane >> 2) & 1;
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            const uint4 qa = *reinterpret_cast<const uint4*>(&tile[tm_sidx<Cfg>(row0 + r, tm_cb<Cfg>(lane, swz))]);
+            const uint4 qb = *reinterpret_cast<const uint4*>(&tile[tm_sidx<Cfg>(row0 + r, tm_cb<Cfg>(lane, swz ^ 1))]);
+            const uint4 q0 = swz ? qb : qa, q1 = swz ? qa : qb;
+            v[r][0] = from_bits<V>(q0.x); v[r][1] = from_bits<V>(q0.y); v[r][2] = from_bits<V>(q0.z);
+            v[r][3] = from_bits<V>(q0.w); v[r][4] = from_bits<V>(q1.x); v[r][5] = from_bits<V>(q1.y);
+            v[r][6] = from_bits<V>(q1.z); v[r][7] = from_bits<V>(q1.w);
+        }
     } else if constexpr (TMA) {
         const TIn* tile = sm.stage[s];
 #pragma unroll
         for (int r = 0; r < RPW; ++r)
 #pragma unroll
             for (int g = 0; g < G; ++g) {
-                const uint4 q = *reinterpret_cast<const uint4*>(&tile[tm_sidx<Cfg>(row0 + r, g * 128 + col0)]);
+                const uint4 q = *reinterpret_cast<const uint4*>(&tile[tm_sidx<Cfg>(row0 + r, tm_cb<Cfg>(lane, g))]);
                 v[r][4 * g] = from_bits<V>(q.x); v[r][4 * g + 1] = from_bits<V>(q.y);
                 v[r][4 * g + 2] = from_bits<V>(q.z); v[r][4 * g + 3] = from_bits<V>(q.w);
             }
@@ -239,7 +260,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
             const long long gi = static_cast<long long>(I) * TR + row0 + r;
 #pragma unroll
             for (int x = 0; x < X; ++x) {
-                const long long gj = static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4);
+                const long long gj = static_cast<long long>(J) * TC + tm_cb<Cfg>(lane, x / 4) + (x % 4);
                 const bool in = gi < p.rows && gj < p.cols;
                 if constexpr (sizeof(TIn) == 1) v[r][x] = in ? V(p.src8[gi * p.src_pitch + gj]) : V(0);
                 else v[r][x] = in ? p.src[gi * p.pitch + gj] : V(0);
@@ -252,7 +273,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
     if (TMA && J == p.C - 1) {  // right edge: zero columns >= cols (16-byte TMA granules, reading R2)
 #pragma unroll
         for (int x = 0; x < X; ++x)
-            if (static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4) >= p.cols) {
+            if (static_cast<long long>(J) * TC + tm_cb<Cfg>(lane, x / 4) + (x % 4) >= p.cols) {
 #pragma unroll
                 for (int r = 0; r < RPW; ++r) v[r][x] = V(0);
             }
@@ -268,7 +289,30 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
     for (int r = 1; r < RPW; ++r)
 #pragma unroll
         for (int x = 0; x < X; ++x) v[r][x] = v[r][x] + v[r - 1][x];
-    if constexpr (G == 1) {
+    if constexpr (Cfg::CT) {
+        // lane-sequential scan of the lane's X contiguous columns, then one warp scan per row (step-major)
+        V incl[RPW];
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+#pragma unroll
+            for (int x = 1; x < X; ++x) v[r][x] = v[r][x] + v[r][x - 1];
+            incl[r] = v[r][X - 1];
+        }
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1)
+#pragma unroll
+            for (int r = 0; r < RPW; ++r) {
+                const V y = __shfl_up_sync(kFull, incl[r], d);
+                if (lane >= d) incl[r] = incl[r] + y;
+            }
+#pragma unroll
+        for (int r = 0; r < RPW; ++r) {
+            V excl = __shfl_up_sync(kFull, incl[r], 1);
+            if (lane == 0) excl = V(0);
+#pragma unroll
+            for (int x = 0; x < X; ++x) v[r][x] = v[r][x] + excl;
+        }
+    } else if constexpr (G == 1) {
 #pragma unroll
         for (int r = 0; r < RPW; ++r) {
             V* w = &v[r][0];
@@ -328,7 +372,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
             named_bar_sync(1, NW * 32);
 #pragma unroll
             for (int g = 0; g < G; ++g)
-                *reinterpret_cast<uint4*>(&bands[warp * TC + g * 128 + col0]) =
+                *reinterpret_cast<uint4*>(&bands[warp * TC + tm_cb<Cfg>(lane, g)]) =
                     make_uint4(to_bits(v[RPW - 1][4 * g]), to_bits(v[RPW - 1][4 * g + 1]),
                                to_bits(v[RPW - 1][4 * g + 2]), to_bits(v[RPW - 1][4 * g + 3]));
             named_bar_sync(1, NW * 32);
@@ -336,7 +380,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
             for (int u = 0; u < warp; ++u)
 #pragma unroll
                 for (int g = 0; g < G; ++g) {
-                    const uint4 q = *reinterpret_cast<const uint4*>(&bands[u * TC + g * 128 + col0]);
+                    const uint4 q = *reinterpret_cast<const uint4*>(&bands[u * TC + tm_cb<Cfg>(lane, g)]);
                     off[4 * g] = off[4 * g] + from_bits<V>(q.x); off[4 * g + 1] = off[4 * g + 1] + from_bits<V>(q.y);
                     off[4 * g + 2] = off[4 * g + 2] + from_bits<V>(q.z);
                     off[4 * g + 3] = off[4 * g + 3] + from_bits<V>(q.w);
@@ -371,7 +415,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
         const uint32_t kind = (I == 0) ? kIncl : kLocal;
 #pragma unroll
         for (int g = 0; g < G; ++g) {
-            uint64_t* cs = p.col_slots + tidx * TC + g * 128 + col0;
+            uint64_t* cs = p.col_slots + tidx * TC + tm_cb<Cfg>(lane, g);
             const V* b = &v[RPW - 1][4 * g];
             st_relaxed2_p(cs, pack(epoch, kind, to_bits(b[0])), pack(epoch, kind, to_bits(b[1])), pol);
             st_relaxed2_p(cs + 2, pack(epoch, kind, to_bits(b[2])), pack(epoch, kind, to_bits(b[3])), pol);
@@ -388,7 +432,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
         if (warp == NW - 1)
 #pragma unroll
             for (int g = 0; g < G; ++g)
-                *reinterpret_cast<uint4*>(&sm.lcs[tq.s][g * 128 + col0]) =
+                *reinterpret_cast<uint4*>(&sm.lcs[tq.s][tm_cb<Cfg>(lane, g)]) =
                     make_uint4(to_bits(v[RPW - 1][4 * g]), to_bits(v[RPW - 1][4 * g + 1]),
                                to_bits(v[RPW - 1][4 * g + 2]), to_bits(v[RPW - 1][4 * g + 3]));
         __syncwarp();
@@ -413,8 +457,8 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
                     if (I > 0) {
 #pragma unroll
                         for (int g = 0; g < G; ++g) {
-                            const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[tq.s][g * 128 + col0]);
-                            uint64_t* cs = p.col_slots + tidx * TC + g * 128 + col0;
+                            const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[tq.s][tm_cb<Cfg>(lane, g)]);
+                            uint64_t* cs = p.col_slots + tidx * TC + tm_cb<Cfg>(lane, g);
                             const V* b = &v[RPW - 1][4 * g];
                             st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(b[0] + from_bits<V>(c4.x))),
                                           pack(epoch, kIncl, to_bits(b[1] + from_bits<V>(c4.y))), pol);
@@ -485,7 +529,7 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
     V cpv[X];
 #pragma unroll
     for (int g = 0; g < G; ++g) {
-        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[q][g * 128 + col0]);
+        const uint4 c4 = *reinterpret_cast<const uint4*>(&sm.cp[q][tm_cb<Cfg>(lane, g)]);
         cpv[4 * g] = from_bits<V>(c4.x); cpv[4 * g + 1] = from_bits<V>(c4.y); cpv[4 * g + 2] = from_bits<V>(c4.z);
         cpv[4 * g + 3] = from_bits<V>(c4.w);
     }
@@ -501,7 +545,7 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
         if (I > 0) {
 #pragma unroll
             for (int g = 0; g < G; ++g) {
-                uint64_t* cs = p.col_slots + tidx * TC + g * 128 + col0;
+                uint64_t* cs = p.col_slots + tidx * TC + tm_cb<Cfg>(lane, g);
                 const V* b = &v[RPW - 1][4 * g];
                 const V* c = &cpv[4 * g];
                 st_relaxed2_p(cs, pack(epoch, kIncl, to_bits(b[0] + c[0])), pack(epoch, kIncl, to_bits(b[1] + c[1])),
@@ -521,7 +565,7 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
     if constexpr (CARRY) {
 #pragma unroll
         for (int x = 0; x < X; ++x) {
-            const long long gj = static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4);
+            const long long gj = static_cast<long long>(J) * TC + tm_cb<Cfg>(lane, x / 4) + (x % 4);
             colterm[x] = colterm[x] + (gj < p.cols ? p.carry[gj] : V(0));
         }
     }
@@ -533,13 +577,17 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
     if (Cfg::DIRECT && !ragged) {
         // Step 4 store straight from registers: a lane writes 16 contiguous bytes of each of its rows
         // (a warp row = 512 contiguous bytes); columns >= cols are clipped, rows >= rows skipped
-        const long long gj = static_cast<long long>(J) * TC + col0;
 #pragma unroll
         for (int r = 0; r < RPW; ++r) {
             const long long gi = static_cast<long long>(I) * TR + row0 + r;
-            if (gi < p.rows && gj < p.cols)
-                __stcs(reinterpret_cast<uint4*>(p.dst + gi * p.pitch + gj),
-                       make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3])));
+#pragma unroll
+            for (int g = 0; g < G; ++g) {
+                const long long gj = static_cast<long long>(J) * TC + tm_cb<Cfg>(lane, g);
+                if (gi < p.rows && gj < p.cols)
+                    __stcs(reinterpret_cast<uint4*>(p.dst + gi * p.pitch + gj),
+                           make_uint4(to_bits(v[r][4 * g]), to_bits(v[r][4 * g + 1]), to_bits(v[r][4 * g + 2]),
+                                      to_bits(v[r][4 * g + 3])));
+            }
         }
     } else if (!ragged) {
         constexpr int WPQ = NW / 4;  // warps per quarter of the buffer
@@ -548,13 +596,24 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
         mbar_wait(&sm.ofree[qq], (ou & 1u) ^ 1u);  // the previous tile's store has read (this quarter of) `out`
         SAT_CLK(o1);
         if (warp == 0 && lane == 0) WS_ST(kWsFastHits, o1 - o0);
+        if constexpr (Cfg::CT) {
+            const int swz = (lane >> 2) & 1;  // same quarter-warp order as the stage read
 #pragma unroll
-        for (int r = 0; r < RPW; ++r)
+            for (int r = 0; r < RPW; ++r) {
+                const uint4 q0 = make_uint4(to_bits(v[r][0]), to_bits(v[r][1]), to_bits(v[r][2]), to_bits(v[r][3]));
+                const uint4 q1 = make_uint4(to_bits(v[r][4]), to_bits(v[r][5]), to_bits(v[r][6]), to_bits(v[r][7]));
+                *reinterpret_cast<uint4*>(&sm.out[tm_sidx<Cfg>(row0 + r, tm_cb<Cfg>(lane, swz))]) = swz ? q1 : q0;
+                *reinterpret_cast<uint4*>(&sm.out[tm_sidx<Cfg>(row0 + r, tm_cb<Cfg>(lane, swz ^ 1))]) = swz ? q0 : q1;
+            }
+        } else {
 #pragma unroll
-            for (int g = 0; g < G; ++g)
-                *reinterpret_cast<uint4*>(&sm.out[tm_sidx<Cfg>(row0 + r, g * 128 + col0)]) =
-                    make_uint4(to_bits(v[r][4 * g]), to_bits(v[r][4 * g + 1]), to_bits(v[r][4 * g + 2]),
-                               to_bits(v[r][4 * g + 3]));
+            for (int r = 0; r < RPW; ++r)
+#pragma unroll
+                for (int g = 0; g < G; ++g)
+                    *reinterpret_cast<uint4*>(&sm.out[tm_sidx<Cfg>(row0 + r, tm_cb<Cfg>(lane, g))]) =
+                        make_uint4(to_bits(v[r][4 * g]), to_bits(v[r][4 * g + 1]), to_bits(v[r][4 * g + 2]),
+                                   to_bits(v[r][4 * g + 3]));
+        }
         fence_proxy_async_smem();
         if constexpr (Cfg::QS) {
             __syncwarp();
@@ -566,7 +625,7 @@ __device__ __forceinline__ void tm_finish(TmSmem<V, Cfg, TIn>& sm, const KParams
             const long long gi = static_cast<long long>(I) * TR + row0 + r;
 #pragma unroll
             for (int x = 0; x < X; ++x) {
-                const long long gj = static_cast<long long>(J) * TC + (x / 4) * 128 + col0 + (x % 4);
+                const long long gj = static_cast<long long>(J) * TC + tm_cb<Cfg>(lane, x / 4) + (x % 4);
                 if (gi < p.rows && gj < p.cols) p.dst[gi * p.pitch + gj] = v[r][x];
             }
         }
