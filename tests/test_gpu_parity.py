@@ -126,6 +126,45 @@ def test_int32_every_variant_and_order(sat, variant, order):
         sat.set_tuning(-1, 0, 0)
 
 
+# production flat-tile kernel (variant 13, 64 x 256 tiles, 2-tile-group order) and its siblings, forced
+# at sizes where auto-selection would pick another kernel: every data path of the ABI contract
+FLAT = [(13, 0x200), (13, 0), (9, 0x200), (17, 0x200), (16, 0)]
+
+
+@pytest.mark.parametrize("variant,order", FLAT)
+def test_flat_tile_kernel_contract(sat, variant, order):
+    sat.set_tuning(variant, order, 0)
+    try:
+        a = satgen.gen_host(700, 1300, seed=71, dist="u32")
+        assert_i32_exact(run_sat(sat, a), a)                        # TMA path, ragged last tile column
+        assert_i32_exact(run_sat(sat, a, pitch=1304), a)            # pitch pad untouched (TMA)
+        assert_i32_exact(run_sat(sat, a, pitch=1301), a)            # generic loads/stores (pitch*4 % 16 != 0)
+        assert_i32_exact(run_sat(sat, a, offset_words=1), a)        # misaligned base: generic path
+        assert_i32_exact(run_sat(sat, a, inplace=True), a)          # src == dst
+        assert_i32_exact(run_sat(sat, a, pitch=1304, inplace=True), a)
+        b = satgen.gen_host(65, 3001, seed=72, dist="u32")         # 2 tile rows, 12 tile columns, ragged both ways
+        assert_i32_exact(run_sat(sat, b, pitch=3004), b)
+        f = satgen.gen_host(1000, 1537, seed=73, dist="fsym")
+        assert_f32_tol(run_sat(sat, f), f)
+        e = satgen.gen_host(640, 2048, seed=74, dist="fu2")         # exact regime: fp32 bit-exact
+        assert (run_sat(sat, e).astype(np.float64) == oracle.sat_f32(e)[0]).all()
+        # carry row (the strip-partitioned path): lower strip of a stacked SAT
+        rows, cols, top = 900, 1100, 357
+        c = satgen.gen_host(rows, cols, seed=75, dist="u32")
+        full = oracle.sat_i32(c)
+        carry = torch.from_numpy(np.ascontiguousarray(full[top - 1])).cuda()
+        assert (run_sat(sat, np.ascontiguousarray(c[top:]), carry=carry) == full[top:]).all()
+        # forward progress with few persistent CTAs
+        for n in [1, 3]:
+            sat.set_max_ctas(n)
+            try:
+                assert_i32_exact(run_sat(sat, a), a)
+            finally:
+                sat.set_max_ctas(0)
+    finally:
+        sat.set_tuning(-1, 0, 0)
+
+
 def test_int32_pitch_pad_untouched(sat):
     a = satgen.gen_host(500, 1000, seed=5, dist="u32")
     assert_i32_exact(run_sat(sat, a, pitch=1024), a)   # TMA path (pitch*4 % 16 == 0)
