@@ -100,6 +100,21 @@ sat_status_t sat_compute(sat_dtype_t dtype, const void* src, void* dst, int64_t 
 sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,
                               int64_t cols, int64_t pitch, void* stream);
 
+/* SATs of a batch of equally shaped matrices in one launch (P:42 per matrix; SURVEY Sec. 8(f)
+ * NEXT-2: many small images, where one matrix has too few tiles to fill 148 SMs):
+ *   dst + k*image_stride = SAT(src + k*image_stride)   for 0 <= k < batch,
+ * each matrix rows x cols with row stride `pitch` elements.  src/dst device; src == dst (in place)
+ * allowed, partial overlap rejected.  image_stride (elements) >= (rows-1)*pitch + cols when
+ * batch > 1.  One CTA per matrix, a single 1R1W pass (column-then-row); meant for
+ * matrices up to ~1K x 1K -- a few large matrices are faster through sat_compute.  16-byte aligned
+ * pointers with pitch and image_stride multiples of 4 take the vector path.  int32 wraps mod 2^32;
+ * fp32 within the tolerance of sat_compute_f32.  Pads are never written.  batch == 0, rows == 0
+ * or cols == 0 is a no-op.
+ * Errors: INVALID_VALUE (sizes, stride, overlap, dtype), MISALIGNED (4-byte), UNSUPPORTED (rows or
+ * cols >= 2^31), CUDA. */
+sat_status_t sat_compute_batched(sat_dtype_t dtype, const void* src, void* dst, int64_t batch, int64_t rows,
+                                 int64_t cols, int64_t pitch, int64_t image_stride, void* stream);
+
 /* ------------------------------------------------------------------ queries on a SAT */
 
 /* Box filter from a SAT b (the O(1) rectangle sum of P:48 that motivates SATs):

@@ -21,7 +21,7 @@ from ._lib import SAT_FLOAT32, SAT_INT32, SatError, SatPlan, check
 _lib.lib()  # load now: fail loudly at import if the native library is missing
 
 __all__ = [
-    "sat", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "sat", "sat_batched", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
     "strip_layout", "broadcast_unique_id",
     "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "release_workspaces",
     "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
@@ -79,6 +79,26 @@ def sat(src, out=None, *, carry=None, stream=None):
         cptr = carry.data_ptr()
     with torch.cuda.device(src.device):
         compute(_dtype_code(src), src.data_ptr(), out.data_ptr(), rows, cols, pitch, cptr, _stream_ptr(stream))
+    return out
+
+
+def sat_batched(src, out=None, *, stream=None):
+    """SATs of a batch of matrices (P:44 per matrix) in one launch: ``src`` is a 3-D int32/float32
+    CUDA tensor (batch, rows, cols) with unit column stride; ``out`` may be ``src`` (in place) or a
+    tensor of the same shape and strides.  For many small matrices."""
+    torch = _torch()
+    if not src.is_cuda or src.dim() != 3 or src.stride(2) != 1:
+        raise ValueError("src: need a 3-D CUDA tensor (batch, rows, cols) with unit column stride")
+    batch, rows, cols = src.shape
+    pitch = src.stride(1) if rows > 1 else max(src.stride(1), cols)
+    stride = src.stride(0) if batch > 1 else max(src.stride(0), (rows - 1) * pitch + cols)
+    if out is None:
+        out = torch.empty_strided(tuple(src.shape), src.stride(), dtype=src.dtype, device=src.device)
+    if out.shape != src.shape or out.stride() != src.stride() or out.dtype != src.dtype or out.device != src.device:
+        raise ValueError("out must match src in shape, strides, dtype and device")
+    with torch.cuda.device(src.device):
+        check(_lib.lib().sat_compute_batched(_dtype_code(src), src.data_ptr(), out.data_ptr(), batch, rows, cols,
+                                             pitch, stride, _stream_ptr(stream)), "sat_compute_batched")
     return out
 
 

@@ -21,6 +21,7 @@
 #include "sat_ws_kernel.cuh"
 #include "sat_tm_kernel.cuh"
 #include "sat_query_kernels.cuh"
+#include "sat_batch_kernel.cuh"
 
 #if defined(SAT_HAVE_NCCL_H)
 #include <nccl.h>
@@ -735,6 +736,61 @@ sat_status_t rects_impl(sat_dtype_t dt, const void* b, int64_t rows, int64_t col
     return SAT_OK;
 }
 
+// ------------------------------------------------------------------ batched small matrices (NEXT-2)
+template <typename V, int NWR>
+cudaError_t launch_batch(bool vec, unsigned grid, const void* src, void* dst, int64_t batch, int64_t rows,
+                         int64_t cols, int64_t pitch, int64_t stride, cudaStream_t st) {
+    const V* a = static_cast<const V*>(src);
+    V* b = static_cast<V*>(dst);
+    constexpr int threads = NWR * 32 * sat::kBatchIpb<NWR>;
+    if (vec) sat::sat_batch_kernel<V, NWR, true><<<grid, threads, 0, st>>>(a, b, batch, rows, cols, pitch, stride);
+    else sat::sat_batch_kernel<V, NWR, false><<<grid, threads, 0, st>>>(a, b, batch, rows, cols, pitch, stride);
+    return cudaGetLastError();
+}
+
+template <typename V>
+cudaError_t launch_batch_w(int nwr, bool vec, unsigned grid, const void* src, void* dst, int64_t batch, int64_t rows,
+                           int64_t cols, int64_t pitch, int64_t stride, cudaStream_t st) {
+    switch (nwr) {
+        case 1: return launch_batch<V, 1>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
+        case 2: return launch_batch<V, 2>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
+        case 4: return launch_batch<V, 4>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
+        default: return launch_batch<V, 8>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
+    }
+}
+
+sat_status_t batched_impl(sat_dtype_t dt, const void* src, void* dst, int64_t batch, int64_t rows, int64_t cols,
+                          int64_t pitch, int64_t stride, cudaStream_t st) {
+    if (dt != SAT_INT32 && dt != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dt);
+    if (batch < 0) return fail(SAT_ERR_INVALID_VALUE, "negative batch");
+    sat_status_t s = validate(batch ? src : nullptr, batch ? dst : nullptr, batch ? rows : 0, cols, pitch);
+    if (s != SAT_OK) return s;
+    if (batch == 0 || rows == 0 || cols == 0) return SAT_OK;
+    const int64_t span = (rows - 1) * pitch + cols;  // elements of one matrix
+    if (batch > 1 && stride < span)
+        return fail(SAT_ERR_INVALID_VALUE, "image_stride %lld < (rows-1)*pitch+cols = %lld (matrices overlap)",
+                    (long long)stride, (long long)span);
+    if (src != dst) {
+        const uintptr_t bytes = static_cast<uintptr_t>(((batch - 1) * stride + span) * 4);
+        const uintptr_t a = reinterpret_cast<uintptr_t>(src), b = reinterpret_cast<uintptr_t>(dst);
+        if (a < b + bytes && b < a + bytes) return fail(SAT_ERR_INVALID_VALUE, "src and dst batches partially overlap");
+    }
+    const bool vec = (((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15u) == 0) &&
+                     (pitch % 4 == 0) && (batch == 1 || stride % 4 == 0);
+    const int nwr = cols <= 128 ? 1 : cols <= 256 ? 2 : cols <= 512 ? 4 : 8;
+    int dev = 0, sms = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    SAT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int64_t cap = static_cast<int64_t>(sms) * 64;  // resident blocks are far fewer; the rest queue
+    const int64_t ctas = nwr == 1 ? (batch + 3) / 4 : batch;  // one-warp CTAs hold 4 matrices (kBatchIpb)
+    const unsigned grid = static_cast<unsigned>(ctas < cap ? ctas : cap);
+    const cudaError_t e = dt == SAT_INT32
+                              ? launch_batch_w<uint32_t>(nwr, vec, grid, src, dst, batch, rows, cols, pitch, stride, st)
+                              : launch_batch_w<float>(nwr, vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
+    if (e != cudaSuccess) return cuda_fail(e, "sat_batch_kernel");
+    return SAT_OK;
+}
+
 // ------------------------------------------------------------------ end-to-end host pipeline
 struct Staging {
     void* buf = nullptr;
@@ -826,6 +882,11 @@ SAT_API sat_status_t sat_box_sum(sat_dtype_t dtype, const void* sat, void* out, 
 SAT_API sat_status_t sat_rect_sums(sat_dtype_t dtype, const void* sat, int64_t rows, int64_t cols, int64_t pitch,
                                    const int64_t* rects, int64_t n, void* out, void* stream) {
     return rects_impl(dtype, sat, rows, cols, pitch, rects, n, out, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_compute_batched(sat_dtype_t dtype, const void* src, void* dst, int64_t batch, int64_t rows,
+                                         int64_t cols, int64_t pitch, int64_t image_stride, void* stream) {
+    return batched_impl(dtype, src, dst, batch, rows, cols, pitch, image_stride, static_cast<cudaStream_t>(stream));
 }
 
 SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,

@@ -55,3 +55,14 @@ cp = med_ms(lambda: out.copy_(t))
 line("i32_sat", med_ms(lambda: sat.sat(t, out=out)), 8, cp)
 line("box_sum_r8", med_ms(lambda: sat.box_sum(t, 8, 8, out=out)), 8, cp)
 line("box_sum_r64", med_ms(lambda: sat.box_sum(t, 64, 64, out=out)), 8, cp)
+# batches of small matrices (sat_compute_batched, one launch) vs the same bytes copied, and vs one
+# sat_compute launch per matrix (timed on the first 256 matrices, scaled to the batch)
+for s in (128, 256, 512, 1024):
+    tb = t.view(-1, s, s)
+    ob = out.view(-1, s, s)
+    ms = med_ms(lambda: sat.sat_batched(tb, out=ob))
+    line(f"batched_{tb.shape[0]}x{s}x{s}_i32", ms, 8, cp)
+    k = 256
+    loop_ms = med_ms(lambda: [sat.sat(tb[i], out=ob[i]) for i in range(k)], reps=3) * tb.shape[0] / k
+    print(json.dumps({"path": f"looped_single_{s}x{s}_i32", "ms_scaled": round(loop_ms, 3),
+                      "batched_speedup": round(loop_ms / ms, 1)}), flush=True)
