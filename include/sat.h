@@ -115,6 +115,20 @@ sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* hos
 sat_status_t sat_compute_batched(sat_dtype_t dtype, const void* src, void* dst, int64_t batch, int64_t rows,
                                  int64_t cols, int64_t pitch, int64_t image_stride, void* stream);
 
+/* Integral images of a batch of 8-bit images (sat_compute_u8 per image, in one launch like
+ * sat_compute_batched): dst + k*image_stride = uint32 SAT of (src + k*src_image_stride).
+ *   src  device u8, row stride src_pitch BYTES (>= cols), image stride src_image_stride BYTES
+ *        (>= (rows-1)*src_pitch + cols when batch > 1).
+ *   dst  device uint32, row stride `pitch` ELEMENTS (>= cols), image stride image_stride ELEMENTS;
+ *        must not overlap src.  Exact while an image's total is < 2^32, modulo 2^32 beyond.
+ * 4-byte aligned src with src_pitch and src_image_stride multiples of 4, and 16-byte aligned dst
+ * with pitch and image_stride multiples of 4, take the vector path.
+ * Errors: INVALID_VALUE (sizes, strides, overlap), MISALIGNED (dst not 4-byte aligned),
+ * UNSUPPORTED (rows or cols >= 2^31), CUDA. */
+sat_status_t sat_compute_batched_u8(const uint8_t* src, int64_t src_pitch, int64_t src_image_stride,
+                                    uint32_t* dst, int64_t batch, int64_t rows, int64_t cols, int64_t pitch,
+                                    int64_t image_stride, void* stream);
+
 /* ------------------------------------------------------------------ queries on a SAT */
 
 /* Box filter from a SAT b (the O(1) rectangle sum of P:48 that motivates SATs):

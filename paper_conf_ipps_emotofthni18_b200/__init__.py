@@ -21,7 +21,7 @@ from ._lib import SAT_FLOAT32, SAT_INT32, SatError, SatPlan, check
 _lib.lib()  # load now: fail loudly at import if the native library is missing
 
 __all__ = [
-    "sat", "sat_batched", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "sat", "sat_batched", "sat_batched_u8", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
     "strip_layout", "broadcast_unique_id",
     "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "release_workspaces",
     "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
@@ -99,6 +99,27 @@ def sat_batched(src, out=None, *, stream=None):
     with torch.cuda.device(src.device):
         check(_lib.lib().sat_compute_batched(_dtype_code(src), src.data_ptr(), out.data_ptr(), batch, rows, cols,
                                              pitch, stride, _stream_ptr(stream)), "sat_compute_batched")
+    return out
+
+
+def sat_batched_u8(src, out=None, *, stream=None):
+    """Integral images of a batch of uint8 images: ``src`` is a 3-D uint8 CUDA tensor (batch, rows, cols)
+    with unit column stride; returns an int32 tensor of the same shape holding the uint32 SATs."""
+    torch = _torch()
+    if src.dtype != torch.uint8 or not src.is_cuda or src.dim() != 3 or src.stride(2) != 1:
+        raise ValueError("src: need a 3-D uint8 CUDA tensor (batch, rows, cols) with unit column stride")
+    batch, rows, cols = src.shape
+    spitch = src.stride(1) if rows > 1 else max(src.stride(1), cols)
+    sstride = src.stride(0) if batch > 1 else max(src.stride(0), (rows - 1) * spitch + cols)
+    if out is None:
+        out = torch.empty((batch, rows, cols), dtype=torch.int32, device=src.device)
+    if out.dtype != torch.int32 or out.device != src.device or out.shape != src.shape or out.stride(2) != 1:
+        raise ValueError("out must be an int32 tensor of src's shape on src's device, unit column stride")
+    pitch = out.stride(1) if rows > 1 else max(out.stride(1), cols)
+    stride = out.stride(0) if batch > 1 else max(out.stride(0), (rows - 1) * pitch + cols)
+    with torch.cuda.device(src.device):
+        check(_lib.lib().sat_compute_batched_u8(src.data_ptr(), spitch, sstride, out.data_ptr(), batch, rows, cols,
+                                                pitch, stride, _stream_ptr(stream)), "sat_compute_batched_u8")
     return out
 
 

@@ -737,26 +737,71 @@ sat_status_t rects_impl(sat_dtype_t dt, const void* b, int64_t rows, int64_t col
 }
 
 // ------------------------------------------------------------------ batched small matrices (NEXT-2)
-template <typename V, int NWR>
+template <typename V, typename TIn, int NWR>
 cudaError_t launch_batch(bool vec, unsigned grid, const void* src, void* dst, int64_t batch, int64_t rows,
-                         int64_t cols, int64_t pitch, int64_t stride, cudaStream_t st) {
-    const V* a = static_cast<const V*>(src);
+                         int64_t cols, int64_t pitch, int64_t stride, int64_t spitch, int64_t sstride, cudaStream_t st) {
+    const TIn* a = static_cast<const TIn*>(src);
     V* b = static_cast<V*>(dst);
     constexpr int threads = NWR * 32 * sat::kBatchIpb<NWR>;
-    if (vec) sat::sat_batch_kernel<V, NWR, true><<<grid, threads, 0, st>>>(a, b, batch, rows, cols, pitch, stride);
-    else sat::sat_batch_kernel<V, NWR, false><<<grid, threads, 0, st>>>(a, b, batch, rows, cols, pitch, stride);
+    if (vec)
+        sat::sat_batch_kernel<V, TIn, NWR, true>
+            <<<grid, threads, 0, st>>>(a, b, batch, rows, cols, pitch, stride, spitch, sstride);
+    else
+        sat::sat_batch_kernel<V, TIn, NWR, false>
+            <<<grid, threads, 0, st>>>(a, b, batch, rows, cols, pitch, stride, spitch, sstride);
     return cudaGetLastError();
 }
 
-template <typename V>
+template <typename V, typename TIn>
 cudaError_t launch_batch_w(int nwr, bool vec, unsigned grid, const void* src, void* dst, int64_t batch, int64_t rows,
-                           int64_t cols, int64_t pitch, int64_t stride, cudaStream_t st) {
+                           int64_t cols, int64_t pitch, int64_t stride, int64_t spitch, int64_t sstride,
+                           cudaStream_t st) {
     switch (nwr) {
-        case 1: return launch_batch<V, 1>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
-        case 2: return launch_batch<V, 2>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
-        case 4: return launch_batch<V, 4>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
-        default: return launch_batch<V, 8>(vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
+        case 1: return launch_batch<V, TIn, 1>(vec, grid, src, dst, batch, rows, cols, pitch, stride, spitch, sstride, st);
+        case 2: return launch_batch<V, TIn, 2>(vec, grid, src, dst, batch, rows, cols, pitch, stride, spitch, sstride, st);
+        case 4: return launch_batch<V, TIn, 4>(vec, grid, src, dst, batch, rows, cols, pitch, stride, spitch, sstride, st);
+        default: return launch_batch<V, TIn, 8>(vec, grid, src, dst, batch, rows, cols, pitch, stride, spitch, sstride, st);
     }
+}
+
+// grid / CTA width of sat_batch_kernel for `batch` matrices of `cols` columns
+int batch_nwr(int64_t cols) { return cols <= 128 ? 1 : cols <= 256 ? 2 : cols <= 512 ? 4 : 8; }
+sat_status_t batch_grid(int64_t batch, int nwr, unsigned* grid) {
+    int dev = 0, sms = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    SAT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int64_t cap = static_cast<int64_t>(sms) * 64;  // resident blocks are far fewer; the rest queue
+    const int64_t ctas = nwr == 1 ? (batch + 3) / 4 : batch;  // one-warp CTAs hold 4 matrices (kBatchIpb)
+    *grid = static_cast<unsigned>(ctas < cap ? ctas : cap);
+    return SAT_OK;
+}
+
+sat_status_t batched_u8_impl(const void* src, int64_t spitch, int64_t sstride, void* dst, int64_t batch, int64_t rows,
+                             int64_t cols, int64_t pitch, int64_t stride, cudaStream_t st) {
+    if (batch < 0 || rows < 0 || cols < 0 || pitch < cols || spitch < cols)
+        return fail(SAT_ERR_INVALID_VALUE, "bad sizes");
+    if (batch == 0 || rows == 0 || cols == 0) return SAT_OK;
+    if (!src || !dst) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    if (reinterpret_cast<uintptr_t>(dst) & 3u) return fail(SAT_ERR_MISALIGNED, "dst must be 4-byte aligned");
+    if (rows > (int64_t(1) << 31) - 1 || cols > (int64_t(1) << 31) - 1)
+        return fail(SAT_ERR_UNSUPPORTED, "rows and cols must be < 2^31");
+    const int64_t span = (rows - 1) * pitch + cols, sspan = (rows - 1) * spitch + cols;
+    if (batch > 1 && (stride < span || sstride < sspan))
+        return fail(SAT_ERR_INVALID_VALUE, "matrix strides smaller than a matrix (matrices overlap)");
+    const uintptr_t a = reinterpret_cast<uintptr_t>(src), b = reinterpret_cast<uintptr_t>(dst);
+    const uintptr_t abytes = static_cast<uintptr_t>((batch - 1) * sstride + sspan);
+    const uintptr_t bbytes = static_cast<uintptr_t>(((batch - 1) * stride + span) * 4);
+    if (a < b + bbytes && b < a + abytes) return fail(SAT_ERR_INVALID_VALUE, "src and dst overlap");
+    const bool vec = ((a & 3u) == 0) && ((b & 15u) == 0) && spitch % 4 == 0 && pitch % 4 == 0 &&
+                     (batch == 1 || (sstride % 4 == 0 && stride % 4 == 0));
+    const int nwr = batch_nwr(cols);
+    unsigned grid = 0;
+    sat_status_t s = batch_grid(batch, nwr, &grid);
+    if (s != SAT_OK) return s;
+    const cudaError_t e =
+        launch_batch_w<uint32_t, uint8_t>(nwr, vec, grid, src, dst, batch, rows, cols, pitch, stride, spitch, sstride, st);
+    if (e != cudaSuccess) return cuda_fail(e, "sat_batch_kernel (u8)");
+    return SAT_OK;
 }
 
 sat_status_t batched_impl(sat_dtype_t dt, const void* src, void* dst, int64_t batch, int64_t rows, int64_t cols,
@@ -777,16 +822,14 @@ sat_status_t batched_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ba
     }
     const bool vec = (((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) & 15u) == 0) &&
                      (pitch % 4 == 0) && (batch == 1 || stride % 4 == 0);
-    const int nwr = cols <= 128 ? 1 : cols <= 256 ? 2 : cols <= 512 ? 4 : 8;
-    int dev = 0, sms = 0;
-    SAT_CUDA(cudaGetDevice(&dev));
-    SAT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    const int64_t cap = static_cast<int64_t>(sms) * 64;  // resident blocks are far fewer; the rest queue
-    const int64_t ctas = nwr == 1 ? (batch + 3) / 4 : batch;  // one-warp CTAs hold 4 matrices (kBatchIpb)
-    const unsigned grid = static_cast<unsigned>(ctas < cap ? ctas : cap);
-    const cudaError_t e = dt == SAT_INT32
-                              ? launch_batch_w<uint32_t>(nwr, vec, grid, src, dst, batch, rows, cols, pitch, stride, st)
-                              : launch_batch_w<float>(nwr, vec, grid, src, dst, batch, rows, cols, pitch, stride, st);
+    const int nwr = batch_nwr(cols);
+    unsigned grid = 0;
+    s = batch_grid(batch, nwr, &grid);
+    if (s != SAT_OK) return s;
+    const cudaError_t e =
+        dt == SAT_INT32
+            ? launch_batch_w<uint32_t, uint32_t>(nwr, vec, grid, src, dst, batch, rows, cols, pitch, stride, pitch, stride, st)
+            : launch_batch_w<float, float>(nwr, vec, grid, src, dst, batch, rows, cols, pitch, stride, pitch, stride, st);
     if (e != cudaSuccess) return cuda_fail(e, "sat_batch_kernel");
     return SAT_OK;
 }
@@ -887,6 +930,13 @@ SAT_API sat_status_t sat_rect_sums(sat_dtype_t dtype, const void* sat, int64_t r
 SAT_API sat_status_t sat_compute_batched(sat_dtype_t dtype, const void* src, void* dst, int64_t batch, int64_t rows,
                                          int64_t cols, int64_t pitch, int64_t image_stride, void* stream) {
     return batched_impl(dtype, src, dst, batch, rows, cols, pitch, image_stride, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_compute_batched_u8(const uint8_t* src, int64_t src_pitch, int64_t src_image_stride,
+                                            uint32_t* dst, int64_t batch, int64_t rows, int64_t cols, int64_t pitch,
+                                            int64_t image_stride, void* stream) {
+    return batched_u8_impl(src, src_pitch, src_image_stride, dst, batch, rows, cols, pitch, image_stride,
+                           static_cast<cudaStream_t>(stream));
 }
 
 SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,

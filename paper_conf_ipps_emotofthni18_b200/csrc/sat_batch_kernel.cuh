@@ -28,18 +28,25 @@ constexpr int kBatchBR = 8;  // rows per band
 template <int NWR>
 constexpr int kBatchIpb = NWR == 1 ? 4 : 1;
 
-// rows [i0, i0 + BR) x columns [j0, j0 + 4) of one matrix; zeros outside it
-template <typename V, bool VEC>
-__device__ __forceinline__ void load_band(V (&v)[kBatchBR][4], const V* a, int64_t i0, int64_t rows, int64_t cols,
+// rows [i0, i0 + BR) x columns [j0, j0 + 4) of one matrix; zeros outside it.  TIn = V (16-byte
+// loads) or uint8_t (u8 pixels, one 32-bit load of 4 pixels, widened to V = uint32).
+template <typename V, typename TIn, bool VEC>
+__device__ __forceinline__ void load_band(V (&v)[kBatchBR][4], const TIn* a, int64_t i0, int64_t rows, int64_t cols,
                                           int64_t pitch, int64_t j0) {
 #pragma unroll
     for (int r = 0; r < kBatchBR; ++r) {
         const int64_t i = i0 + r;
-        const V* p = a + i * pitch + j0;
+        const TIn* p = a + i * pitch + j0;
         if (VEC && i < rows && j0 + 3 < cols) {
-            const uint4 q = *reinterpret_cast<const uint4*>(p);
-            v[r][0] = from_bits<V>(q.x); v[r][1] = from_bits<V>(q.y);
-            v[r][2] = from_bits<V>(q.z); v[r][3] = from_bits<V>(q.w);
+            if constexpr (sizeof(TIn) == 1) {
+                const uint32_t w = *reinterpret_cast<const uint32_t*>(p);
+#pragma unroll
+                for (int x = 0; x < 4; ++x) v[r][x] = V((w >> (8 * x)) & 0xffu);
+            } else {
+                const uint4 q = *reinterpret_cast<const uint4*>(p);
+                v[r][0] = from_bits<V>(q.x); v[r][1] = from_bits<V>(q.y);
+                v[r][2] = from_bits<V>(q.z); v[r][3] = from_bits<V>(q.w);
+            }
         } else {
 #pragma unroll
             for (int x = 0; x < 4; ++x) v[r][x] = (i < rows && j0 + x < cols) ? p[x] : V(0);
@@ -47,10 +54,11 @@ __device__ __forceinline__ void load_band(V (&v)[kBatchBR][4], const V* a, int64
     }
 }
 
-template <typename V, int NWR, bool VEC>
-__global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>) sat_batch_kernel(const V* src, V* dst, int64_t batch,
+// src: matrices of TIn with row stride spitch / matrix stride sstride; dst: V with pitch / stride
+template <typename V, typename TIn, int NWR, bool VEC>
+__global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>) sat_batch_kernel(const TIn* src, V* dst, int64_t batch,
                                                             int64_t rows, int64_t cols, int64_t pitch,
-                                                            int64_t stride) {
+                                                            int64_t stride, int64_t spitch, int64_t sstride) {
     constexpr int BR = kBatchBR, CW = 128 * NWR;
     __shared__ V wtot[2][NWR][BR];
     constexpr int IPB = kBatchIpb<NWR>;
@@ -58,17 +66,18 @@ __global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>) sat_batch_kernel(co
     const int64_t first = static_cast<int64_t>(blockIdx.x) * IPB + (IPB > 1 ? threadIdx.x >> 5 : 0);
     int par = 0;
     for (int64_t img = first; img < batch; img += static_cast<int64_t>(gridDim.x) * IPB) {
-        const V* a = src + img * stride;
+        const TIn* a = src + img * sstride;
         V* b = dst + img * stride;
         for (int64_t c0 = 0; c0 < cols; c0 += CW) {
             const int64_t j0 = c0 + warp * 128 + lane * 4;  // this lane's first column
             V carry[4] = {V(0), V(0), V(0), V(0)};         // c_{i0 - 1}[j0 .. j0 + 3]
-            // 8-warp CTAs (few, wide matrices) load the next band one band ahead so that its loads
-            // overlap this band's scans; narrower CTAs are numerous enough to hide the latency and run
-            // faster without the extra registers (measured)
-            constexpr bool PF = NWR >= 8;
+            // 8-warp CTAs (few, wide matrices) and u8 inputs (only 128 B per warp row in flight) load
+            // the next band one band ahead so that its loads overlap this band's scans; narrower int32 /
+            // fp32 CTAs are numerous enough to hide the latency and run faster without the extra
+            // registers (measured)
+            constexpr bool PF = NWR >= 8 || sizeof(TIn) == 1;
             V nx[BR][4];
-            if (PF) load_band<V, VEC>(nx, a, 0, rows, cols, pitch, j0);
+            if (PF) load_band<V, TIn, VEC>(nx, a, 0, rows, cols, spitch, j0);
             for (int64_t i0 = 0; i0 < rows; i0 += BR) {
                 V v[BR][4];
                 if (PF) {
@@ -76,9 +85,9 @@ __global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>) sat_batch_kernel(co
                     for (int r = 0; r < BR; ++r)
 #pragma unroll
                         for (int x = 0; x < 4; ++x) v[r][x] = nx[r][x];
-                    if (i0 + BR < rows) load_band<V, VEC>(nx, a, i0 + BR, rows, cols, pitch, j0);
+                    if (i0 + BR < rows) load_band<V, TIn, VEC>(nx, a, i0 + BR, rows, cols, spitch, j0);
                 } else {
-                    load_band<V, VEC>(v, a, i0, rows, cols, pitch, j0);
+                    load_band<V, TIn, VEC>(v, a, i0, rows, cols, spitch, j0);
                 }
                 // left term b[i][c0 - 1] (0 for the first chunk); written by this CTA one chunk earlier
                 V left[BR];

@@ -145,3 +145,64 @@ def test_batched_edge_cases(sat):
     assert lib.sat_compute_batched(0, x.data_ptr(), x.data_ptr(), -1, 4, 8, 8, 32, None) == 1
     assert lib.sat_compute_batched(0, x.data_ptr(), x.data_ptr(), 1, 4, 8, 7, 32, None) == 1
     assert lib.sat_compute_batched(9, x.data_ptr(), x.data_ptr(), 1, 4, 8, 8, 32, None) == 1
+
+
+# ---------------------------------------------------------------- u8 images -> uint32 integral images
+
+def make_u8(batch, rows, cols, seed):
+    return make_batch(batch, rows, cols, dist="u8", seed=seed).astype(np.uint8)
+
+
+def run_u8(sat, img, spitch=None, sstride=None, soff=0, pitch=None, stride=None):
+    batch, rows, cols = img.shape
+    spitch = cols if spitch is None else spitch
+    sstride = rows * spitch if sstride is None else sstride
+    pitch = cols if pitch is None else pitch
+    stride = rows * pitch if stride is None else stride
+    n = (batch - 1) * sstride + (rows - 1) * spitch + cols
+    sbuf = torch.full((n + soff + 16,), 0xA5, dtype=torch.uint8, device="cuda")
+    src = torch.as_strided(sbuf, (batch, rows, cols), (sstride, spitch, 1), soff)
+    src.copy_(torch.from_numpy(np.ascontiguousarray(img)).cuda())
+    m = (batch - 1) * stride + (rows - 1) * pitch + cols
+    obuf = torch.full((m + 16,), SENTINEL, dtype=torch.int32, device="cuda")
+    out = torch.as_strided(obuf, (batch, rows, cols), (stride, pitch, 1))
+    sat.sat_batched_u8(src, out=out)
+    torch.cuda.synchronize()
+    mask = torch.ones_like(obuf, dtype=torch.bool)
+    torch.as_strided(mask, (batch, rows, cols), (stride, pitch, 1)).fill_(False)
+    assert (obuf[mask] == SENTINEL).all(), "words outside the integral images were written"
+    return out.cpu().numpy()
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 1), (5, 9, 9), (4, 100, 128), (3, 65, 129), (3, 200, 256),
+                                   (2, 129, 513), (2, 300, 1024), (2, 50, 2047)])
+def test_batched_u8_parity(sat, shape):
+    img = make_u8(*shape, seed=900 + shape[2])
+    got = run_u8(sat, img)
+    for k in range(shape[0]):
+        assert (got[k] == oracle.sat_i32(img[k].astype(np.int32))).all(), f"image {k}"
+
+
+@pytest.mark.parametrize("spitch,sstride,soff,pitch", [(130, None, 0, None), (128, 128 * 40 + 4, 0, 132),
+                                                       (128, None, 1, None), (131, 131 * 40 + 5, 3, 129)])
+def test_batched_u8_layouts(sat, spitch, sstride, soff, pitch):
+    img = make_u8(4, 40, 127, seed=17)
+    got = run_u8(sat, img, spitch=spitch, sstride=sstride, soff=soff, pitch=pitch)
+    for k in range(4):
+        assert (got[k] == oracle.sat_i32(img[k].astype(np.int32))).all()
+
+
+def test_batched_u8_wraps_mod_2_32(sat):
+    # all-255 images whose totals pass 2^31 and 2^32: the uint32 bit pattern (mod 2^32)
+    img = np.full((2, 3000, 6000), 255, dtype=np.uint8)
+    got = run_u8(sat, img)
+    i, j = np.arange(3000)[:, None] + 1, np.arange(6000)[None, :] + 1
+    want = ((i * j * 255) % (1 << 32)).astype(np.uint32).view(np.int32)
+    assert (got[0] == want).all() and (got[1] == want).all()
+
+
+def test_batched_u8_matches_single(sat):
+    img = make_u8(3, 333, 1500, seed=23)
+    got = run_u8(sat, img)
+    for k in range(3):
+        assert (sat.sat_u8(torch.from_numpy(img[k].copy()).cuda()).cpu().numpy() == got[k]).all()

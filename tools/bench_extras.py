@@ -66,3 +66,9 @@ for s in (128, 256, 512, 1024):
     loop_ms = med_ms(lambda: [sat.sat(tb[i], out=ob[i]) for i in range(k)], reps=3) * tb.shape[0] / k
     print(json.dumps({"path": f"looped_single_{s}x{s}_i32", "ms_scaled": round(loop_ms, 3),
                       "batched_speedup": round(loop_ms / ms, 1)}), flush=True)
+# batched u8 -> uint32 integral images (1 B read + 4 B written per pixel) vs the widening copy
+img = t.to(torch.uint8)
+cp5 = med_ms(lambda: out.copy_(img))
+for s in (256, 1024):
+    ms = med_ms(lambda: sat.sat_batched_u8(img.view(-1, s, s), out=out.view(-1, s, s)))
+    line(f"batched_u8_{n * n // (s * s)}x{s}x{s}", ms, 5, cp5)
