@@ -56,7 +56,14 @@ __device__ __forceinline__ void load_band(V (&v)[kBatchBR][4], const TIn* a, int
 
 // src: matrices of TIn with row stride spitch / matrix stride sstride; dst: V with pitch / stride
 template <typename V, typename TIn, int NWR, bool VEC>
-__global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>) sat_batch_kernel(const TIn* src, V* dst, int64_t batch,
+// >= 768 resident threads per SM (<= 85 registers) for the narrow CTAs and for u8 input: unbounded,
+// ptxas used 130-190 registers there and left 10-14 warps per SM (ncu: 12% warps active for u8
+// 256 x 256).  The 8-warp int32 / fp32 CTAs get 2 CTAs per SM (<= 128 registers): the one-band-ahead
+// loads spill under the 85-register cap (1024^2: +19.5% over copy) and 150 unbounded registers leave
+// one CTA per SM (+22.6%); at 128 registers +4.9% (measured)
+__global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>,
+                                  (sizeof(TIn) == 1 || NWR < 8) ? 768 / (NWR * 32 * kBatchIpb<NWR>) : 2)
+    sat_batch_kernel(const TIn* src, V* dst, int64_t batch,
                                                             int64_t rows, int64_t cols, int64_t pitch,
                                                             int64_t stride, int64_t spitch, int64_t sstride) {
     constexpr int BR = kBatchBR, CW = 128 * NWR;
@@ -71,11 +78,10 @@ __global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>) sat_batch_kernel(co
         for (int64_t c0 = 0; c0 < cols; c0 += CW) {
             const int64_t j0 = c0 + warp * 128 + lane * 4;  // this lane's first column
             V carry[4] = {V(0), V(0), V(0), V(0)};         // c_{i0 - 1}[j0 .. j0 + 3]
-            // 8-warp CTAs (few, wide matrices) and u8 inputs (only 128 B per warp row in flight) load
-            // the next band one band ahead so that its loads overlap this band's scans; narrower int32 /
-            // fp32 CTAs are numerous enough to hide the latency and run faster without the extra
-            // registers (measured)
-            constexpr bool PF = NWR >= 8 || sizeof(TIn) == 1;
+            // 8-warp CTAs (few, wide matrices) load the next band one band ahead so that its loads
+            // overlap this band's scans; narrower CTAs are numerous enough to hide the latency and run
+            // faster without the extra registers (measured)
+            constexpr bool PF = NWR >= 8;
             V nx[BR][4];
             if (PF) load_band<V, TIn, VEC>(nx, a, 0, rows, cols, spitch, j0);
             for (int64_t i0 = 0; i0 < rows; i0 += BR) {
