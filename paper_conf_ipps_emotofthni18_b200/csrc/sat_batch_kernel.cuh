@@ -54,6 +54,27 @@ __device__ __forceinline__ void load_band(V (&v)[kBatchBR][4], const TIn* a, int
     }
 }
 
+// u8 pixels of rows [i0, i0 + BR) x columns [j0, j0 + 4) as raw 32-bit words (pixel x in byte x);
+// zeros outside the matrix.  Prefetching these costs BR registers instead of 4 BR.
+template <bool VEC>
+__device__ __forceinline__ void load_words_u8(uint32_t (&w)[kBatchBR], const uint8_t* a, int64_t i0, int64_t rows,
+                                              int64_t cols, int64_t pitch, int64_t j0) {
+#pragma unroll
+    for (int r = 0; r < kBatchBR; ++r) {
+        const int64_t i = i0 + r;
+        const uint8_t* p = a + i * pitch + j0;
+        if (VEC && i < rows && j0 + 3 < cols) {
+            w[r] = *reinterpret_cast<const uint32_t*>(p);
+        } else {
+            uint32_t x = 0;
+#pragma unroll
+            for (int c = 0; c < 4; ++c)
+                if (i < rows && j0 + c < cols) x |= static_cast<uint32_t>(p[c]) << (8 * c);
+            w[r] = x;
+        }
+    }
+}
+
 // src: matrices of TIn with row stride spitch / matrix stride sstride; dst: V with pitch / stride
 template <typename V, typename TIn, int NWR, bool VEC>
 // >= 768 resident threads per SM (<= 85 registers) for the narrow CTAs and for u8 input: unbounded,
@@ -79,14 +100,25 @@ __global__ void __launch_bounds__(NWR * 32 * kBatchIpb<NWR>,
             const int64_t j0 = c0 + warp * 128 + lane * 4;  // this lane's first column
             V carry[4] = {V(0), V(0), V(0), V(0)};         // c_{i0 - 1}[j0 .. j0 + 3]
             // 8-warp CTAs (few, wide matrices) load the next band one band ahead so that its loads
-            // overlap this band's scans; narrower CTAs are numerous enough to hide the latency and run
-            // faster without the extra registers (measured)
+            // overlap this band's scans; narrower int32 / fp32 CTAs are numerous enough to hide the
+            // latency and run faster without the extra registers (measured).  u8
+            // input always loads one band ahead, as raw words (8 registers; a warp row is only 128 B)
             constexpr bool PF = NWR >= 8;
-            V nx[BR][4];
-            if (PF) load_band<V, TIn, VEC>(nx, a, 0, rows, cols, spitch, j0);
+            constexpr bool U8 = sizeof(TIn) == 1;
+            V nx[PF && !U8 ? BR : 1][4];
+            uint32_t nw[U8 ? BR : 1];
+            if constexpr (U8) load_words_u8<VEC>(nw, reinterpret_cast<const uint8_t*>(a), 0, rows, cols, spitch, j0);
+            else if constexpr (PF) load_band<V, TIn, VEC>(nx, a, 0, rows, cols, spitch, j0);
             for (int64_t i0 = 0; i0 < rows; i0 += BR) {
                 V v[BR][4];
-                if (PF) {
+                if constexpr (U8) {
+#pragma unroll
+                    for (int r = 0; r < BR; ++r)
+#pragma unroll
+                        for (int x = 0; x < 4; ++x) v[r][x] = V((nw[r] >> (8 * x)) & 0xffu);
+                    if (i0 + BR < rows)
+                        load_words_u8<VEC>(nw, reinterpret_cast<const uint8_t*>(a), i0 + BR, rows, cols, spitch, j0);
+                } else if constexpr (PF) {
 #pragma unroll
                     for (int r = 0; r < BR; ++r)
 #pragma unroll
