@@ -105,3 +105,34 @@ def test_strip_bounds_cover_rows_exactly(sat):
             for r0, n in parts:
                 assert n >= 0 and (n == 0 or r0 == pos)
                 pos += n
+
+
+def test_batched_argument_validation_without_gpu(sat):
+    """sat_compute_batched / _u8 reject bad arguments before any CUDA call (include/sat.h)."""
+    from paper_conf_ipps_emotofthni18_b200 import _lib
+
+    L = _lib.lib()
+    B = L.sat_compute_batched
+    assert B(0, None, None, 0, 5, 5, 5, 25, None) == 0  # empty batch: no-op, null pointers allowed
+    assert B(1, None, None, 3, 0, 5, 5, 25, None) == 0  # empty matrices
+    assert B(0, 16, 16, -1, 4, 8, 8, 32, None) == 1  # negative batch
+    assert B(0, 16, 16, 2, 4, 8, 7, 32, None) == 1  # pitch < cols
+    assert B(5, 16, 16, 2, 4, 8, 8, 32, None) == 1  # unknown dtype
+    assert B(0, 16, 16, 2, 4, 8, 8, 31, None) == 1  # image stride < (rows-1)*pitch + cols
+    assert b"overlap" in L.sat_last_error_detail()
+    assert B(0, 18, 1 << 20, 2, 4, 8, 8, 32, None) == 2  # misaligned
+    assert B(0, 1 << 20, (1 << 20) + 64, 2, 4, 8, 8, 32, None) == 1  # batches partially overlap
+    U = L.sat_compute_batched_u8
+    assert U(None, 8, 32, None, 0, 4, 8, 8, 32, None) == 0
+    assert U(16, 7, 32, 1 << 20, 2, 4, 8, 8, 32, None) == 1  # src_pitch < cols
+    assert U(16, 8, 31, 1 << 20, 2, 4, 8, 8, 32, None) == 1  # src image stride too small
+    assert U(16, 8, 32, (1 << 20) + 2, 2, 4, 8, 8, 32, None) == 2  # dst misaligned
+    assert U(1 << 20, 8, 32, (1 << 20) + 8, 2, 4, 8, 8, 32, None) == 1  # src and dst overlap
+
+
+def test_batched_binding_rejects_bad_tensors(sat):
+    torch = pytest.importorskip("torch")
+    with pytest.raises(ValueError):
+        sat.sat_batched(torch.zeros(2, 3, 4, dtype=torch.int32))  # not a CUDA tensor
+    with pytest.raises(ValueError):
+        sat.sat_batched_u8(torch.zeros(2, 3, 4, dtype=torch.uint8))
