@@ -18,7 +18,6 @@
 #include "sat.h"
 #include "sat_aux_kernels.cuh"
 #include "sat_kernel.cuh"
-#include "sat_ws_kernel.cuh"
 #include "sat_tm_kernel.cuh"
 #include "sat_query_kernels.cuh"
 #include "sat_batch_kernel.cuh"
@@ -88,6 +87,7 @@ struct Family<sat::TileCfg<TR, TC, NW, ST>> {
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_tiles_kernel<V, Cfg, TMA, CARRY>); }
 };
 
+#if SAT_EXPERIMENTAL
 template <int TR, int NW, int ST, int NT, int NQ, int FLAGS>
 struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
     using Cfg = sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>;
@@ -98,6 +98,8 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
     template <typename V, bool TMA, bool CARRY>
     static void* kernel() { return reinterpret_cast<void*>(&sat::sat_ws_kernel<V, Cfg, TMA, CARRY>); }
 };
+
+#endif
 
 template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC, int LB, int CT>
 struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT>> {
@@ -210,26 +212,32 @@ Variant make_variant() {
     return v;
 }
 
+// Shipped kernel variants (auto_variant picks among them; sat_set_tuning can force one, test hook).
+// Tuning builds (-DSAT_EXPERIMENTAL=1) append the configurations measured and not kept in round 1
+// (DESIGN.md Sec. 5), so that they can still be re-measured.
+enum : int { kVarClassic = 0, kVarTm128 = 1, kVarU8 = 2, kVarFlat = 3 };
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
-        make_variant<sat::TmCfg<16, 2, 5>>(),  // 0: local SAT parked in TMEM, 2 input stages + output buffer, walkers publish
-        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 1: deferred finish, GSAT from registers
-        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch>>(),  // 2: 64 KiB tiles, 3 stages, TMA store
-        make_variant<sat::TmCfg<16, 2, 5, 1, 2>>(),  // 3: TMEM-parked, walkers publish (blocking on the local aggregates)
-        make_variant<sat::TileCfg<64, 128, 8, 2>>(),   // 4: classic, 32 KiB tiles, 2 stages
-        make_variant<sat::TileCfg<128, 128, 16, 2>>(), // 5: classic, 64 KiB tiles, 512 threads
-        make_variant<sat::TmCfg<16, 2, 7, 1, 1, 4>>(),  // 6: experimental
-        make_variant<sat::TmCfg<16, 3, 8, 1, 3, 4, 1>>(),  // 7
-        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 8
-        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),  // 9
-        make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>>(),  // 10: u8 integral images only (4 stages of 16 KiB u8 tiles)
-        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),    // 11: flat 64 x 256 tiles, 8 compute warps, ring of 8
-        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 64, 256>>(),    // 12: ... ring of 7
-        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 13: ... ring of 6
-        make_variant<sat::TmCfg<8, 2, 10, 1, 3, 4, 0, 0, 64, 256>>(),   // 14: ... ring of 10
-        make_variant<sat::TmCfg<16, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),   // 15: 16 compute warps (4 rows each)
-        make_variant<sat::TmCfg<8, 3, 7, 1, 3, 4, 1, 0, 64, 256>>(),    // 16: GSAT stored from registers, 3 stages
-        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 1>>(),  // 17: variant 13, lanes own 8 contiguous columns
+        make_variant<sat::TileCfg<64, 128, 8, 2>>(),                   // 0: classic, 64 x 128 tiles (small matrices)
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),                  // 1: TMEM-parked, 128 x 128 tiles
+        make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>>(),                  // 2: u8 integral images (4 stages of 16 KiB)
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 3: TMEM-parked, flat 64 x 256 tiles
+#if SAT_EXPERIMENTAL
+        make_variant<sat::TmCfg<16, 2, 5>>(),  // 4: walkers publish (blocking ws_walker)
+        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 5
+        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch>>(),  // 6: warp-specialised, TMA store
+        make_variant<sat::TmCfg<16, 2, 5, 1, 2>>(),  // 7
+        make_variant<sat::TileCfg<128, 128, 16, 2>>(),  // 8: classic, 128 x 128 tiles
+        make_variant<sat::TmCfg<16, 2, 7, 1, 1, 4>>(),  // 9
+        make_variant<sat::TmCfg<16, 3, 8, 1, 3, 4, 1>>(),  // 10: GSAT from registers
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 11
+        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),    // 12: flat, ring of 8
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 64, 256>>(),    // 13: flat, ring of 7
+        make_variant<sat::TmCfg<8, 2, 10, 1, 3, 4, 0, 0, 64, 256>>(),   // 14: flat, ring of 10
+        make_variant<sat::TmCfg<16, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),   // 15: flat, 16 compute warps
+        make_variant<sat::TmCfg<8, 3, 7, 1, 3, 4, 1, 0, 64, 256>>(),    // 16: flat, GSAT from registers
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 1>>(),  // 17: flat, 8 contiguous columns
+#endif
     };
     return vs;
 }
@@ -247,14 +255,14 @@ int auto_variant(int64_t rows, int64_t cols) {
     // latency; above, the TMEM-parked kernel with decoupled walkers (parking depth 4) on flat
     // 64 x 256 tiles
     const int64_t n = rows * cols;
-    return n <= (int64_t(1) << 21) ? 4 : (n <= (int64_t(1) << 25) ? 9 : 13);
+    return n <= (int64_t(1) << 21) ? kVarClassic : (n <= (int64_t(1) << 25) ? kVarTm128 : kVarFlat);
 }
 
 int auto_order(int vi, int64_t cols) {
     // flat 64 x 256 tiles with >= 128 tile columns (>= 32K columns): anti-diagonal order of 2-wide tile
     // groups (each DRAM row visit 2 KiB); narrower grids keep the plain anti-diagonal order, which
     // measured faster there (tools/sweep_variants.py, profiles/r01_sweep_sizes.jsonl)
-    return (vi == 13 && (cols + 255) / 256 >= 128) ? 0x200 : 0;
+    return (vi == kVarFlat && (cols + 255) / 256 >= 128) ? 0x200 : 0;
 }
 
 // ------------------------------------------------------------------ device info caches
@@ -464,7 +472,7 @@ sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* sr
     int vi, order;
     {
         std::lock_guard<std::mutex> lk(g_mu);
-        vi = g_variant >= 0 ? g_variant : (u8 ? 10 : auto_variant(rows, cols));
+        vi = g_variant >= 0 ? g_variant : (u8 ? kVarU8 : auto_variant(rows, cols));
         order = (g_variant < 0 && g_order == 0) ? auto_order(vi, cols) : g_order;
     }
     const Variant& v = variants()[vi];

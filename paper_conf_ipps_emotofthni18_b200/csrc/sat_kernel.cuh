@@ -38,6 +38,10 @@ constexpr uint32_t kEpochMax = (1u << 30) - 1u;
 #ifndef SAT_STATS
 #define SAT_STATS 0
 #endif
+// Tuning builds (-DSAT_EXPERIMENTAL=1): the kernel configurations measured in round 1 and not shipped.
+#ifndef SAT_EXPERIMENTAL
+#define SAT_EXPERIMENTAL 0
+#endif
 constexpr int kNumStats = 24;
 enum StatSlot {
     kStTiles = 0, kStLoop, kStTicket, kStFullWait, kStCompute, kStRowLb, kStRowSteps, kStRowSpins, kStColLb,

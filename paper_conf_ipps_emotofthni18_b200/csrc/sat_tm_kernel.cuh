@@ -1,10 +1,10 @@
 // sat_tm_kernel.cuh -- single-pass SAT kernel for sm_100a with the local SAT parked in tensor memory.
 //
-// Same method, aggregates and walkers as sat_ws_kernel (1R1W-SKSS-LB of PAPER.md Sec. IV, P:182-249,
-// prefix-form slots, epoch-tagged status words; walkers: ws_walker).  What differs is where a tile
-// waits for its look-backs.  In sat_ws_kernel the compute warps hold a tile's local SAT in registers
-// and its input stage in shared memory until the walks land (~1 us per tile on B200 with HBM
-// saturated), which idles the warps and pins a 64 KiB stage.  Here:
+// The method is 1R1W-SKSS-LB of PAPER.md Sec. IV with prefix-form slots and epoch-tagged
+// status words (sat_kernel.cuh).  What this kernel is built around is where a tile waits for its
+// look-backs: with HBM saturated a look-back round trip costs ~1 us on B200, so a compute warp that
+// held its tile until the walks land would idle and pin a 64 KiB stage (the superseded warp-
+// specialised sat_ws_kernel, now only in -DSAT_EXPERIMENTAL tuning builds).  Here:
 //
 //   * a tile's pixels are read out of their input stage into registers right away and the stage is
 //     handed back to the loader (the ring refills while the tile is still being computed);
@@ -22,7 +22,10 @@
 // of each of its waiters.
 #pragma once
 
-#include "sat_ws_kernel.cuh"
+#include "sat_pipe.cuh"
+#if SAT_EXPERIMENTAL
+#include "sat_ws_kernel.cuh"  // ws_walker (non-decoupled walker configurations, tuning builds only)
+#endif
 
 namespace sat {
 
@@ -64,6 +67,9 @@ struct TmCfg {
     static_assert(!CT || (TC == 256 && !DIRECT), "contiguous lane columns: 64 x 256 tiles");
     static_assert(D >= 2 && D * TM_COLS_PER_SLOT <= 512, "TMEM columns");
     static_assert(IN >= 1 && NQ >= IN + D - 1 && NQ <= 16, "rings");
+#if !SAT_EXPERIMENTAL
+    static_assert(DECOUPLED, "product builds ship the decoupled walkers only (-DSAT_EXPERIMENTAL=1 for the rest)");
+#endif
 };
 
 template <typename V, typename Cfg, typename TIn = V>
@@ -887,11 +893,17 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         named_bar_sync(2, NW * 32);
         if (warp == 0) tmem_dealloc(sm.tmem_base, Cfg::TM_COLS);
     } else if (warp == Cfg::ROW_WARP) {
-        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, true, TIn>(sm, p, epoch, lane);
-        else ws_walker<V, Cfg, true>(sm, p, epoch, lane);
+#if SAT_EXPERIMENTAL
+        if constexpr (!Cfg::DECOUPLED) ws_walker<V, Cfg, true>(sm, p, epoch, lane);
+        else
+#endif
+        tm_walker<V, Cfg, true, TIn>(sm, p, epoch, lane);
     } else if (warp == Cfg::COL_WARP) {
-        if constexpr (Cfg::DECOUPLED) tm_walker<V, Cfg, false, TIn>(sm, p, epoch, lane);
-        else ws_walker<V, Cfg, false>(sm, p, epoch, lane);
+#if SAT_EXPERIMENTAL
+        if constexpr (!Cfg::DECOUPLED) ws_walker<V, Cfg, false>(sm, p, epoch, lane);
+        else
+#endif
+        tm_walker<V, Cfg, false, TIn>(sm, p, epoch, lane);
     } else if (warp == Cfg::STORE_WARP) {
         // ================================================================ storer (one lane)
         if (lane == 0) {

@@ -126,9 +126,10 @@ def test_int32_every_variant_and_order(sat, variant, order):
         sat.set_tuning(-1, 0, 0)
 
 
-# production flat-tile kernel (variant 13, 64 x 256 tiles, 2-tile-group order) and its siblings, forced
-# at sizes where auto-selection would pick another kernel: every data path of the ABI contract
-FLAT = [(13, 0x200), (13, 0), (9, 0x200), (17, 0x200), (16, 0)]
+# production flat-tile kernel (variant 3, 64 x 256 tiles, 2-tile-group order) and the 128 x 128 kernel
+# (variant 1), forced at sizes where auto-selection would pick another kernel: every data path of the
+# ABI contract
+FLAT = [(3, 0x200), (3, 0), (1, 0x200), (1, 0)]
 
 
 @pytest.mark.parametrize("variant,order", FLAT)
