@@ -16,12 +16,14 @@ Contents (PAPER.md cited as P:<line>; readings R<n> are listed in DESIGN.md):
   each written as the region sum that defines it.
 * ``tile_order`` -- the diagonal-major serial numbering of Fig. 9 (R6).
 * ``rect_sum`` -- the rectangle query of P:48; ``box_sum`` -- the box filter built from it.
-* ``strip_carry_u32`` / ``strip_carry_f64`` -- the carry row of a horizontal strip (column sums of
-  all rows above it), read from the streaming state (R12, multi-GPU).
+* ``strip_carry_u32`` -- the carry row of a horizontal strip (column sums of all rows above it), read
+  from the streaming state (R12, multi-GPU); ``Stream.colsums_f64`` is its fp64 counterpart.
+* ``moments_f32`` -- the two SATs of a summed-area variance shadow map, SAT(a) and SAT(a*a) (P:50 and
+  its ref. [8]), in fp64 from fp32 input, with their absSATs.
 * ``f32_tolerance`` -- the fp32 acceptance bound of BASELINE.json north_star (R10).
 
-Every function is pinned by tests/test_oracle.py against something other than itself; none is
-"parity unpinned".
+Every function is pinned by tests/test_oracle.py against something other than itself (the test
+named after each function is listed in DESIGN.md Sec. 3); none is "parity unpinned".
 """
 from __future__ import annotations
 
@@ -134,6 +136,17 @@ def sat_f64(a: np.ndarray) -> np.ndarray:
     return b
 
 
+def moments_f32(a: np.ndarray):
+    """Summed-area variance shadow map moments (ref. [8] P:311): the SAT of a and the SAT of
+    a*a, both by the column-then-row passes of P:46 in fp64 (a fp32 value squares exactly in fp64),
+    each with its absSAT for the R10 tolerance.  Returns (sat1, abs1, sat2, abs2); abs2 == sat2."""
+    a = np.ascontiguousarray(a, dtype=np.float32)
+    s1, ab1 = sat_f32(a)
+    sq = a.astype(np.float64) * a.astype(np.float64)
+    s2 = sat_f64(sq)
+    return s1, ab1, s2, s2.copy()
+
+
 # ------------------------------------------------------------------------------------ streaming
 class Stream:
     """Streaming oracle: feed input rows top to bottom, get SAT rows back (O(cols) state)."""
@@ -194,14 +207,21 @@ def region_sum(a: np.ndarray, U: int, D: int, L: int, R: int):
 
 
 def rect_sum(b: np.ndarray, u: int, d: int, l: int, r: int):
-    """sum of a[i][j] for u < i <= d, l < j <= r, from four SAT entries (uint32 arithmetic).
-    Index -1 denotes the empty prefix (SAT value 0)."""
-    def at(i, j):
-        return 0 if (i < 0 or j < 0) else int(b[i, j])
+    """sum of a[i][j] for u < i <= d, l < j <= r, from four SAT entries; index -1 denotes the
+    empty prefix (SAT value 0).  Evaluated in b's own arithmetic, left to right as P:48 writes it,
+    ((b[d][r] - b[u][r]) - b[d][l]) + b[u][l] (reading R17): uint32 wraparound for integer b (an int),
+    fp32 for float32 b (an np.float32), fp64 for float64 b."""
+    if b.dtype in (np.uint32, np.int32):
+        def at(i, j):
+            return 0 if (i < 0 or j < 0) else int(b[i, j]) % (1 << 32)
 
-    if b.dtype == np.uint32 or b.dtype == np.int32:
-        return (at(d, r) - at(u, r) - at(d, l) + at(u, l)) % (1 << 32)
-    return at(d, r) - at(u, r) - at(d, l) + at(u, l)
+        return (((at(d, r) - at(u, r)) - at(d, l)) + at(u, l)) % (1 << 32)
+    z = b.dtype.type(0)
+
+    def atf(i, j):
+        return z if (i < 0 or j < 0) else b[i, j]
+
+    return ((atf(d, r) - atf(u, r)) - atf(d, l)) + atf(u, l)
 
 
 def box_sum(b: np.ndarray, rh: int, rw: int) -> np.ndarray:

@@ -35,7 +35,9 @@
  *
  * Parity pins for every function here live in tests/test_oracle.py (brute force over
  * the P:44 definition, Figure 2 golden tables, rectangle formula P:48, closed forms,
- * invariants).  No function in this file is "parity unpinned".
+ * invariants); DESIGN.md Sec. 3 lists the pin of each function, including
+ * oracle_region_sum_f64 (test_region_sum_f64_against_fsum).  No function in this file
+ * is "parity unpinned".
  */
 #include <math.h>
 #include <stdint.h>

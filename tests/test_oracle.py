@@ -305,3 +305,85 @@ def test_f32_tolerance_accepts_fp32_sat_and_rejects_perturbation():
     bad = f32.astype(np.float64).copy()
     bad[150, 100] += 4 * tol[150, 100] + 1e-3
     assert not (np.abs(bad - b) <= tol).all()
+
+
+# ----------------------------------------------------------------------------- fp32 / fp64 branches
+def test_region_sum_f64_against_fsum():
+    """oracle_region_sum_f64 (S[U:D][L:R] of P:128 for float input) vs the exactly rounded sum."""
+    a = (RNG.random((11, 14), dtype=np.float32) * 2 - 1).astype(np.float32)
+    rows, cols = a.shape
+    for U, D in itertools.combinations_with_replacement(range(rows), 2):
+        for L, R in [(0, cols - 1), (3, 3), (2, 9), (13, 13), (5, 12)]:
+            blk = a[U:D + 1, L:R + 1].astype(np.float64).ravel()
+            got = oracle.region_sum(a, U, D, L, R)
+            assert abs(got - math.fsum(blk)) <= blk.size * 2.0 ** -53 * math.fsum(np.abs(blk)) + 1e-300
+    assert oracle.region_sum(a, 5, 4, 0, 3) == 0.0  # empty range (D < U): the zero aggregates of R5
+    assert oracle.region_sum(a, 0, 3, 7, 6) == 0.0
+    # integers below 2^24 (exact in fp32 and in every fp64 partial): equals the integer region sum
+    ai = RNG.integers(-(2 ** 20), 2 ** 20, size=(9, 10)).astype(np.float32)
+    assert oracle.region_sum(ai, 2, 7, 1, 8) == float(ai[2:8, 1:9].astype(np.int64).sum())
+
+
+def test_rect_sum_float_branches():
+    """rect_sum on float32 / float64 SATs: the P:48 formula in the SAT's own precision (R17)."""
+    a = RNG.integers(0, 4, size=(9, 12)).astype(np.float64)
+    b64 = oracle.sat_f64(a)  # exact: small integers
+    b32 = b64.astype(np.float32)
+    rows, cols = a.shape
+    for u, d in itertools.combinations(range(-1, rows), 2):
+        for l, r in itertools.combinations(range(-1, cols), 2):
+            want = float(a[u + 1: d + 1, l + 1: r + 1].sum())
+            g32 = oracle.rect_sum(b32, u, d, l, r)
+            assert isinstance(g32, np.float32) and float(g32) == want
+            assert oracle.rect_sum(b64, u, d, l, r) == want
+    # association: ((drr - urr) - dll) + ull, each step rounded to fp32
+    bf = (RNG.standard_normal((6, 7)) * 1e4).astype(np.float32)
+    want = ((bf[5, 6] - bf[2, 6]) - bf[5, 3]) + bf[2, 3]
+    assert oracle.rect_sum(bf, 2, 5, 3, 6) == want
+    assert oracle.rect_sum(bf, -1, 5, -1, 6) == bf[5, 6]
+
+
+def test_table2_float_branch_against_fsum():
+    """Table II of an fp32 matrix (fp64 region sums): every entry within the fp64 summation bound of
+    the exactly rounded region sum, and the P:162 / P:233 / P:241 relations to fp64 rounding."""
+    a = (RNG.random((10, 13), dtype=np.float32) * 2 - 1).astype(np.float32)
+    TR, TC = 4, 5
+    rows, cols = a.shape
+    eps = 64 * 2.0 ** -53 * float(np.abs(a.astype(np.float64)).sum())
+    fs = lambda U, D, L, R: math.fsum(a[U:D + 1, L:R + 1].astype(np.float64).ravel()) if (D >= U and R >= L) else 0.0  # noqa: E731
+    T = {(I, J): oracle.table2(a, TR, TC, I, J) for I in range(3) for J in range(3)}
+    for (I, J), t in T.items():
+        r0, c0 = TR * I, TC * J
+        r1, c1 = min(r0 + TR, rows) - 1, min(c0 + TC, cols) - 1
+        assert abs(t["GS"] - fs(0, r1, 0, c1)) <= eps
+        assert abs(t["LS"] - fs(r0, r1, c0, c1)) <= eps
+        assert abs(t["GLS"] - (fs(0, r1, 0, c1) - fs(0, r0 - 1, 0, c0 - 1))) <= eps  # the L-shaped region
+        for i in range(r1 - r0 + 1):
+            assert abs(t["GRS"][i] - fs(r0 + i, r0 + i, 0, c1)) <= eps
+            assert abs(t["LRS"][i] - fs(r0 + i, r0 + i, c0, c1)) <= eps
+        for j in range(c1 - c0 + 1):
+            assert abs(t["GCS"][j] - fs(0, r1, c0 + j, c0 + j)) <= eps
+        gs_d = T[(I - 1, J - 1)]["GS"] if (I > 0 and J > 0) else 0.0
+        assert abs(t["GS"] - (gs_d + t["GLS"])) <= eps  # Step 3.3
+        grs_l = T[(I, J - 1)]["GRS"] if J > 0 else [0.0] * len(t["LRS"])
+        assert all(abs(t["GRS"][i] - (grs_l[i] + t["LRS"][i])) <= eps for i in range(len(t["LRS"])))  # P:233
+
+
+def test_moments_f32_against_fsum_and_closed_form():
+    """Variance-shadow-map moments (ref. [8]): SAT(a) and SAT(a*a) vs exactly rounded sums; a
+    constant c gives (i+1)(j+1)c and (i+1)(j+1)c^2."""
+    a = (RNG.random((13, 17), dtype=np.float32) * 2 - 1).astype(np.float32)
+    s1, ab1, s2, ab2 = oracle.moments_f32(a)
+    a64 = a.astype(np.float64)
+    for i in range(a.shape[0]):
+        for j in range(a.shape[1]):
+            blk = a64[: i + 1, : j + 1].ravel()
+            sq = blk * blk
+            assert abs(s1[i, j] - math.fsum(blk)) <= (i + j + 2) * 2.0 ** -52 * math.fsum(np.abs(blk))
+            assert abs(ab1[i, j] - math.fsum(np.abs(blk))) <= (i + j + 2) * 2.0 ** -52 * math.fsum(np.abs(blk))
+            assert abs(s2[i, j] - math.fsum(sq)) <= (i + j + 2) * 2.0 ** -52 * math.fsum(sq)
+    assert (ab2 == s2).all()
+    c = np.full((6, 9), 0.75, dtype=np.float32)
+    i, j = np.indices(c.shape)
+    s1, _, s2, _ = oracle.moments_f32(c)
+    assert (s1 == (i + 1) * (j + 1) * 0.75).all() and (s2 == (i + 1) * (j + 1) * 0.5625).all()
