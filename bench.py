@@ -102,11 +102,35 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------------- CPU baseline (oracle)
-def cpu_oracle_sample(rows: int, cols: int, dtype: str, target_s: float = 12.0) -> dict:
-    """Time the CPU oracle (oracle/, as it stands, single thread) on a bounded sample of the workload:
-    the first `h` rows (all columns) of the same seeded matrix, h chosen for ~target_s of CPU work."""
-    import numpy as np
+def host_cpu() -> dict:
+    model = "unknown"
+    try:
+        for ln in Path("/proc/cpuinfo").read_text().splitlines():
+            if ln.startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count()}
 
+
+class pinned_to_one_core:
+    """Run the single-threaded oracle pinned to one host core (sched_setaffinity), then restore."""
+
+    def __enter__(self):
+        self.prev = os.sched_getaffinity(0)
+        self.core = min(self.prev)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.prev)
+
+
+def cpu_oracle_sample(rows: int, cols: int, dtype: str, target_s: float = 12.0) -> dict:
+    """Time the CPU oracle (oracle/, as it stands, single thread pinned to one core) on a bounded sample
+    of the workload: the first `h` rows (all columns) of the same seeded matrix, h chosen for ~target_s of
+    CPU work."""
     import oracle
     import satgen
 
@@ -121,18 +145,21 @@ def cpu_oracle_sample(rows: int, cols: int, dtype: str, target_s: float = 12.0) 
             oracle.sat_u32(a)
         return time.perf_counter() - t0
 
-    h = min(rows, 64)
-    t = run(h)
-    while t < 0.5 and h < rows:
-        h = min(rows, h * 4)
+    with pinned_to_one_core() as pin:
+        h = min(rows, 64)
         t = run(h)
-    rate = h * cols / t
-    h2 = int(min(rows, max(h, rate * target_s / cols)))
-    if h2 > h:
-        h, t = h2, run(h2)
+        while t < 0.5 and h < rows:
+            h = min(rows, h * 4)
+            t = run(h)
+        rate = h * cols / t
+        h2 = int(min(rows, max(h, rate * target_s / cols)))
+        if h2 > h:
+            h, t = h2, run(h2)
+        core = pin.core
     return {"value": h * cols / t / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"first {h} of {rows} rows x {cols} cols ({dtype}, seed 1447), in-memory oracle "
-                      f"(column-then-row, single thread), {t:.2f} s", "_np": np.__version__}
+            "sample": f"first {h} of {rows} rows x {cols} cols ({dtype}, seed 1447), in-memory C oracle "
+                      f"(column-then-row, single thread pinned to core {core}), {t:.2f} s",
+            **host_cpu()}
 
 
 # ------------------------------------------------------------------------------------- helpers
@@ -145,15 +172,19 @@ def order_name(order: int) -> str:
 
 
 def load_ncu_traffic(workload: str):
+    """DRAM read + write bytes per launch of this workload's SAT kernel from the committed ncu capture
+    (profiles/ncu_summary.json, one `ncu --set full` launch of the same kernel and configuration)."""
     p = ROOT / "profiles" / "ncu_summary.json"
     if not p.exists():
-        return None
+        return None, None
     try:
         d = json.loads(p.read_text())
         e = d.get(workload)
-        return None if e is None else e.get("dram_bytes_per_launch")
+        if e is None:
+            return None, None
+        return e.get("dram_bytes_per_launch"), f"profiles/ncu_summary.json ({e.get('source', 'ncu --set full')})"
     except Exception:
-        return None
+        return None, None
 
 
 def dist_info():
@@ -181,22 +212,24 @@ def run_reference(args):
     h = max(1, min(rows, int(os.environ.get("SAT_REF_ROWS", "2048"))))
     a = satgen.gen_host(h, cols, 1447, dist)
     f = (lambda: oracle.sat_f32(a, with_abs=False)) if dtype == "f32" else (lambda: oracle.sat_u32(a))
-    for _ in range(args.warmup):
-        f()
     times = []
-    for _ in range(args.steps):
-        t0 = time.perf_counter()
-        f()
-        times.append(time.perf_counter() - t0)
+    with pinned_to_one_core():
+        for _ in range(args.warmup):
+            f()
+        for _ in range(args.steps):
+            t0 = time.perf_counter()
+            f()
+            times.append(time.perf_counter() - t0)
     ms = statistics.mean(times) * 1e3
     value = h * cols / (ms / 1e3) / 1e9
-    sample = f"first {h} of {rows} rows x {cols} cols per step ({dtype}, seed 1447), single-thread C oracle"
+    sample = (f"first {h} of {rows} rows x {cols} cols per step ({dtype}, seed 1447), single-thread C oracle "
+              f"pinned to one core")
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak" if world == 1 else "strong",
         "vs_baseline": None, "dtype": "f64" if dtype == "f32" else "u32", "data": "synthetic",
         "config": {"workload": f"{n}x{n} {dtype} SAT (sampled rows)", "rows": rows, "cols": cols},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample, **host_cpu()},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
         "gpu_launches": 0,
     }
@@ -217,6 +250,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--sweep", action="store_true")
+    ap.add_argument("--no-extras", action="store_true", help="skip the other BASELINE configs (4K^2, sweep, 64K^2)")
     ap.add_argument("--variant", type=int, default=-1)
     ap.add_argument("--order", type=int, default=0)
     ap.add_argument("--ctas-per-sm", type=int, default=0)
@@ -314,19 +348,7 @@ def main():
     # ---- end to end through the C ABI with host buffers (rank 0 of N=1 only; PCIe-bound)
     e2e = None
     if rank == 0 and world == 1 and not args.no_e2e:
-        h_in = torch.empty((rows, cols), dtype=tdt, pin_memory=True)
-        h_out = torch.empty((rows, cols), dtype=tdt, pin_memory=True)
-        h_in.copy_(x)
-        sat.sat_host(h_in.numpy(), h_out.numpy())  # warm-up (allocates the staging buffer)
-        t0 = time.perf_counter()
-        for _ in range(args.e2e_steps):
-            sat.sat_host(h_in.numpy(), h_out.numpy())
-        e2e_s = (time.perf_counter() - t0) / args.e2e_steps
-        ok = bool(torch.equal(h_out[-1, -8:].to(dev), y[-1, -8:])) if args.dtype == "i32" else True
-        e2e = {"value": total_elems / e2e_s / 1e9, "unit": UNIT, "h2d_bytes_per_step": total_elems * 4,
-               "d2h_bytes_per_step": total_elems * 4, "ms_per_step": e2e_s * 1e3,
-               "path": "sat_compute_host (pinned host buffers; strip-pipelined H2D | SAT | D2H)", "check": ok}
-        del h_in, h_out
+        e2e = run_e2e(args, sat, torch, x, rows, cols, tdt)
 
     if rank == 0:
         peak, peak_src = measured_peaks()
@@ -335,6 +357,7 @@ def main():
         workload = f"{n}x{n} {args.dtype} SAT" + ("" if world == 1 else f" strip-partitioned over {world} GPUs")
         plan = sat.query_plan(sat.SAT_FLOAT32 if args.dtype == "f32" else sat.SAT_INT32, nrows, cols, cols,
                               x.data_ptr(), y.data_ptr())
+        traffic, traffic_src = load_ncu_traffic(workload)
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
@@ -349,24 +372,179 @@ def main():
                        "parallelism": "single GPU" if world == 1 else f"strips x{world}"},
             "hbm_gbs": achieved,
             "memcpy": {"ms": memcpy_ms, "gbs": nrows * cols * BYTES_PER_ELEM / (memcpy_ms / 1e3) / 1e9,
-                       "overhead_pct": (ms - memcpy_ms) / memcpy_ms * 100.0},
+                       "overhead_pct": (ms - memcpy_ms) / memcpy_ms * 100.0, "ratio": ms / memcpy_ms,
+                       "gate": "<= 1.10 x memcpy (BASELINE north_star)"},
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": load_ncu_traffic(workload), "peak_source": peak_src,
-                         "kernel": {2: "sat_tm_kernel", 1: "sat_ws_kernel"}.get(plan["family"], "sat_tiles_kernel"),
-                         "bytes_per_elem": BYTES_PER_ELEM},
+                         "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
+                         "peak_source": peak_src,
+                         "kernel": {2: "sat_tm_kernel"}.get(plan["family"], "sat_tiles_kernel"),
+                         "bytes_per_elem": BYTES_PER_ELEM,
+                         "timing": "CUDA events on the launching stream around the K timed launches"},
             "gpu_launches": args.steps * (1 if world == 1 else 4),
             "clocks": clk,
             "e2e": e2e,
         }
+        if world == 1 and not args.no_extras:
+            del y
+            line["extras"] = run_extras(args, sat, satgen, torch, x, peak)
         if world == 1 and not args.no_cpu:
-            cb = cpu_oracle_sample(rows, cols, args.dtype)
-            cb.pop("_np", None)
-            line["cpu_baseline"] = cb
+            line["cpu_baseline"] = cpu_oracle_sample(rows, cols, args.dtype)
         print(json.dumps(line), flush=True)
     if comm is not None:
         comm.close()
         dist.destroy_process_group()
     return 0
+
+
+# ------------------------------------------------------------------------------------- e2e (host buffers)
+def run_e2e(args, sat, torch, x, rows, cols, tdt) -> dict:
+    """The public host-buffer call (sat_compute_host): pinned input, H2D + SAT + D2H inside the timed
+    region, then a sampled check of the result against the oracle (first 64 rows exactly as computed by
+    the streaming oracle, and the last row after feeding the oracle every row of the input)."""
+    import numpy as np
+
+    import oracle
+
+    h_in = torch.empty((rows, cols), dtype=tdt, pin_memory=True)
+    h_out = torch.empty((rows, cols), dtype=tdt, pin_memory=True)
+    h_in.copy_(x)
+    # PCIe roofline: plain pinned copies of the same bytes, each direction alone
+    dbuf = torch.empty_like(x)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    dbuf.copy_(h_in, non_blocking=True)
+    torch.cuda.synchronize()
+    h2d_s = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    h_out.copy_(dbuf, non_blocking=True)
+    torch.cuda.synchronize()
+    d2h_s = time.perf_counter() - t0
+    del dbuf
+    nbytes = rows * cols * 4
+    sat.sat_host(h_in.numpy(), h_out.numpy())  # warm-up (allocates the staging buffer)
+    t0 = time.perf_counter()
+    for _ in range(args.e2e_steps):
+        sat.sat_host(h_in.numpy(), h_out.numpy())
+    e2e_s = (time.perf_counter() - t0) / args.e2e_steps
+    a = h_in.numpy()
+    got = h_out.numpy()
+    st = oracle.Stream(cols)
+    if a.dtype == np.int32:
+        head_ok = bool((got[:64] == st.rows_u32(a[:64]).view(np.int32)).all())
+        st.rows_u32(a[64:rows - 1], want_out=False)
+        tail_ok = bool((got[rows - 1:] == st.rows_u32(a[rows - 1:]).view(np.int32)).all())
+    else:
+        w, ab = st.rows_f32(a[:64])
+        head_ok = bool((np.abs(got[:64] - w) <= oracle.f32_tolerance(ab, rows, cols)).all())
+        st.rows_f32(a[64:rows - 1], want_out=False, want_abs=False)
+        w, ab = st.rows_f32(a[rows - 1:])
+        tail_ok = bool((np.abs(got[rows - 1:] - w) <= oracle.f32_tolerance(ab, rows, cols)).all())
+    st.close()
+    h2d_gbs, d2h_gbs = nbytes / h2d_s / 1e9, nbytes / d2h_s / 1e9
+    # the copies in and out overlap with each other and with the SAT; the bound is the slower direction
+    pcie_floor_s = max(nbytes / (h2d_gbs * 1e9), nbytes / (d2h_gbs * 1e9))
+    return {"value": rows * cols / e2e_s / 1e9, "unit": UNIT, "h2d_bytes_per_step": nbytes,
+            "d2h_bytes_per_step": nbytes, "ms_per_step": e2e_s * 1e3,
+            "path": "sat_compute_host (pinned host buffers; strip-pipelined H2D | SAT | D2H)",
+            "pcie": {"h2d_gbs": h2d_gbs, "d2h_gbs": d2h_gbs, "floor_ms": pcie_floor_s * 1e3,
+                     "frac_of_floor": pcie_floor_s / e2e_s,
+                     "how": "one pinned torch copy of the same bytes per direction, wall clock"},
+            "check": {"first_64_rows": head_ok, "last_row": tail_ok,
+                      "how": "streaming oracle over every input row; int32 bit-exact, fp32 R10 tolerance"}}
+
+
+# ------------------------------------------------------------------------------------- extras
+def graph_time(torch, fn, per_graph=20, reps=5) -> float:
+    """Device ms per call: `per_graph` calls captured in one CUDA graph (no host launch cost), best of
+    `reps` replays timed with CUDA events on the replay stream."""
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            fn()
+    torch.cuda.current_stream().wait_stream(s)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(per_graph):
+            fn()
+    g.replay()
+    torch.cuda.synchronize()
+    best = 1e30
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        g.replay()
+        e1.record()
+        torch.cuda.synchronize()
+        best = min(best, e0.elapsed_time(e1) / per_graph)
+    del g
+    return best
+
+
+def event_time(torch, fn, reps) -> float:
+    """Device ms per call: `reps` back-to-back launches between two CUDA events (after 3 warm-ups)."""
+    for _ in range(3):
+        fn()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps):
+        fn()
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps
+
+
+def size_point(torch, sat, satgen, n, dtype, peak, rows=None) -> dict:
+    rows = rows or n
+    x = torch.empty((rows, n), dtype=torch.int32, device="cuda")
+    satgen.fill_tensor(x, 1447, "f01" if dtype == "f32" else "u32")
+    if dtype == "f32":
+        x = x.view(torch.float32)
+    y = torch.empty_like(x)
+    if rows * n <= (1 << 26):  # latency-bound sizes: device time through CUDA graphs
+        t_sat = graph_time(torch, lambda: sat.sat(x, out=y))
+        t_cp = graph_time(torch, lambda: y.copy_(x))
+        how = "CUDA graph of 20 calls, best of 5 replays"
+    else:
+        reps = max(10, min(200, int(4e10 / (rows * n * 8))))
+        t_sat = event_time(torch, lambda: sat.sat(x, out=y), reps)
+        t_cp = event_time(torch, lambda: y.copy_(x), reps)
+        how = f"{reps} back-to-back launches between CUDA events"
+    gbs = rows * n * BYTES_PER_ELEM / (t_sat / 1e3) / 1e9
+    plan = sat.query_plan(sat.SAT_FLOAT32 if dtype == "f32" else sat.SAT_INT32, rows, n)
+    del x, y
+    return {"rows": rows, "cols": n, "dtype": dtype, "sat_ms": t_sat, "memcpy_ms": t_cp,
+            "overhead_pct": (t_sat - t_cp) / t_cp * 100.0, "gelems": rows * n / (t_sat / 1e3) / 1e9,
+            "gbs": gbs, "frac": gbs / peak, "tile": [plan["tile_rows"], plan["tile_cols"]], "timing": how}
+
+
+def run_extras(args, sat, satgen, torch, x, peak) -> dict:
+    """Every other BASELINE.json config on this GPU in the same run (device time, same-run memcpy):
+    configs[1] 4K^2 int32/fp32, configs[2] the paper's size sweep 256^2..32K^2 int32 (Table III analogue,
+    overhead over duplication per size), int32 32K^2, and configs[4]'s 64K^2 int32 as
+    a single pass on one GPU (the 'linear' baseline of the strip-partitioned scaling)."""
+    del x
+    torch.cuda.empty_cache()
+    out = {}
+    out["c1_4k"] = {d: size_point(torch, sat, satgen, 4096, d, peak) for d in ("i32", "f32")}
+    out["i32_32k"] = size_point(torch, sat, satgen, 32768, "i32", peak)
+    out["sweep_i32"] = [size_point(torch, sat, satgen, 1 << k, "i32", peak) for k in range(8, 16)]
+    # 64K^2 int32 single GPU, in place (16 GiB) against a 16 GiB copy
+    n = 65536
+    xx = torch.empty((n, n), dtype=torch.int32, device="cuda")
+    satgen.fill_tensor(xx, 1447, "u32")
+    t_sat = event_time(torch, lambda: sat.sat(xx, out=xx), 5)
+    yy = torch.empty_like(xx)
+    t_cp = event_time(torch, lambda: yy.copy_(xx), 5)
+    del xx, yy
+    torch.cuda.empty_cache()
+    gbs = n * n * BYTES_PER_ELEM / (t_sat / 1e3) / 1e9
+    out["i32_64k_single_gpu"] = {"rows": n, "cols": n, "sat_ms": t_sat, "memcpy_ms": t_cp,
+                                 "overhead_pct": (t_sat - t_cp) / t_cp * 100.0, "gbs": gbs, "frac": gbs / peak,
+                                 "note": "in place; 5 launches between CUDA events"}
+    return out
 
 
 def run_sweep(args, sat, satgen, torch):

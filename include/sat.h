@@ -29,8 +29,13 @@
  *     deterministic.  fp32: IEEE adds in an unspecified, run-dependent association; every entry
  *     satisfies |dst - exact| <= (rows+cols) * 1.2e-7 * SAT(|src|) at that entry (R10).
  *   - libsat owns its workspace (per-tile aggregates, status words, tile counter), cached per
- *     (device, stream) and grown on demand with cudaMalloc; growth is the only synchronising
- *     event and must not happen inside CUDA-graph capture (call once before capturing).
+ *     (device, stream) and grown on demand, stream-ordered (cudaMallocAsync / cudaFreeAsync on
+ *     that stream, no host synchronisation); the first call on a new (device, stream) resets the
+ *     workspace's control block synchronously, so call once before capturing a CUDA graph.
+ *     sat_release_stream_workspace frees one stream's workspace (e.g. before destroying the stream),
+ *     sat_release_workspaces all of them.
+ *   - Thread safety: calls on different streams run concurrently; calls on the same stream from
+ *     several host threads are serialised per workspace.  sat_compute_host is serialised per device.
  */
 #ifndef LIBSAT_SAT_H
 #define LIBSAT_SAT_H
@@ -96,7 +101,9 @@ sat_status_t sat_compute(sat_dtype_t dtype, const void* src, void* dst, int64_t 
  * strips (H2D of strip k+1, SAT of strip k and D2H of strip k-1 overlap; strip k uses the last SAT
  * row of strip k-1 as its carry row).  host_src/host_dst: rows x cols, row stride `pitch`
  * elements, may be the same buffer; pinned memory gives full PCIe bandwidth.  Device staging
- * buffers are owned by libsat (cached per device).  Synchronous. */
+ * buffers, copy streams and events are owned by libsat (cached per device); concurrent calls on one
+ * device are serialised (a per-device lock held until the call's final synchronisation).
+ * Synchronous. */
 sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, void* host_dst, int64_t rows,
                               int64_t cols, int64_t pitch, void* stream);
 
@@ -177,7 +184,10 @@ sat_status_t sat_comm_destroy(sat_comm_t comm);
  * order on every rank with equal `cols`.  Rank r passes ITS horizontal strip: global rows
  * [row0_r, row0_r + strip_rows) with row0_r = sum of strip_rows of ranks < r (strips may differ in
  * height).  Steps: sat_strip_colsum -> ncclAllGather of the colsum vectors -> sat_carry_prefix ->
- * sat_compute with that carry.  strip_src/strip_dst device (this rank), may be equal. */
+ * sat_compute with that carry.  strip_src/strip_dst device (this rank), may be equal.
+ * Errors: a null comm, unknown dtype or cols <= 0 (arguments equal on every rank) return before the
+ * collective; a rank-local failure (bad strip_rows / pitch, overlap, misalignment, column-sum launch)
+ * still joins the all-gather with a zero vector, so no other rank blocks, and is then returned. */
 sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, const void* strip_src,
                                  void* strip_dst, int64_t strip_rows, int64_t cols, int64_t pitch,
                                  void* stream);
@@ -193,7 +203,7 @@ typedef struct {
     int64_t aux_bytes;     /* bytes of per-tile aggregate slots for this shape */
     int32_t variant;       /* kernel variant index */
     int32_t order;         /* 0 = diagonal-major (Fig. 9), 1 = row-major */
-    int32_t family;        /* 1 = warp-specialised kernel (sat_ws_kernel), 0 = classic (sat_tiles_kernel) */
+    int32_t family;        /* 2 = TMEM-parked kernel (sat_tm_kernel), 0 = classic (sat_tiles_kernel) */
     int32_t reserved;
 } sat_plan_t;
 
@@ -201,9 +211,12 @@ typedef struct {
 sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t cols, int64_t pitch,
                             const void* src, const void* dst, sat_plan_t* plan);
 
-/* Tuning knobs (process-wide; for sweeps and tests).  variant: -1 = automatic choice;
- * order: 0 = diagonal-major (Fig. 9), 1 = row-major; ctas_per_sm: 0 = occupancy maximum.
- * Returns INVALID_VALUE for an unknown variant. */
+/* TEST / TUNING HOOKS (process-wide; for sweeps and tests -- not part of the computing API).
+ * variant: -1 = automatic choice, else an index < sat_num_variants() (the shipped library has the
+ * four variants auto-selection uses: 0 classic 64x128, 1 TMEM-parked 128x128, 2 u8 integral images,
+ * 3 TMEM-parked flat 64x256; -DSAT_EXPERIMENTAL builds append the unshipped tuning configurations);
+ * order: 0 = diagonal-major (Fig. 9), 1 = row-major, (g << 8) = diagonal-major over g-tile
+ * groups; ctas_per_sm: 0 = occupancy maximum.  Returns INVALID_VALUE for an unknown variant. */
 sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm);
 int sat_num_variants(void);
 /* Cap the total number of persistent CTAs (0 = no cap).  A cap of 1 runs the whole matrix on one
@@ -226,6 +239,24 @@ sat_status_t sat_debug_stats(int64_t* out, int max_ctas, int* n_ctas, int* n_sta
  * aggregates published, 3 row walk resolved, 4 column walk resolved, 5 Step 4 done, 6 store issued,
  * 7 TMA load issued (0 where a step does not apply to the variant). */
 sat_status_t sat_debug_trace(int64_t* out, int64_t max_tiles, int64_t* n_tiles);
+
+/* Test hook: the published aggregate words of the most recent sat_compute launch on (current
+ * device, `stream`) -- the per-tile slots of Steps 2.A/2.B/3 in their final state.
+ * info (required) receives the tile grid; host_out (NULL = only fill info) receives info->words
+ * 64-bit status words (synchronises `stream`): row slots [R*C][tile_rows], column slots
+ * [R*C][tile_cols], corner slots [R*C], tile t = I*C + J.  A word is (epoch << 34 | kind << 32 |
+ * value bits), kind 1 = local, 2 = inclusive; row / column slots hold prefix sums over the tile's
+ * rows / columns (R5'), the corner GLS (local) or GS (inclusive).  Classic-kernel launches
+ * (small matrices) share the layout.  Errors: INVALID_VALUE (no workspace, max_words too small), CUDA. */
+typedef struct {
+    int32_t tile_rows, tile_cols, R, C;
+    int64_t words;
+} sat_ws_info_t;
+sat_status_t sat_debug_workspace(void* stream, uint64_t* host_out, int64_t max_words, sat_ws_info_t* info);
+
+/* Free the cached workspace of (current device, `stream`) (synchronises the stream); a later call
+ * on that stream allocates a new one.  Call before destroying a stream libsat has used. */
+sat_status_t sat_release_stream_workspace(void* stream);
 
 /* Free every cached workspace and staging buffer (synchronises the devices that own them). */
 sat_status_t sat_release_workspaces(void);

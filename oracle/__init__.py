@@ -250,9 +250,10 @@ def box_sum(b: np.ndarray, rh: int, rw: int) -> np.ndarray:
 
 
 # ------------------------------------------------------------------------------------ Table II
-def table2(a: np.ndarray, TR: int, TC: int, I: int, J: int) -> dict:
+def table2(a: np.ndarray, TR: int, TC: int, I: int, J: int, with_gsat: bool = True) -> dict:
     """The per-tile sums of Table II for tile T(I,J) of TR x TC tiles (reading R5), each computed
-    as the region sum S[..][..] that defines it.  Rows/cols beyond the matrix are absent (zero)."""
+    as the region sum S[..][..] that defines it.  Rows/cols beyond the matrix are absent (zero).
+    ``with_gsat=False`` skips GSAT (TR*TC region sums) for large tiles."""
     rows, cols = a.shape
     r0, c0 = TR * I, TC * J
     r1, c1 = min(r0 + TR, rows) - 1, min(c0 + TC, cols) - 1
@@ -267,7 +268,8 @@ def table2(a: np.ndarray, TR: int, TC: int, I: int, J: int) -> dict:
         # GLS(I,J): the L-shaped region [0:r1] x [0:c1] minus [0:r0-1] x [0:c0-1] (Fig. 11 caption)
         "GLS": (S(r0, r1, 0, c1) + S(0, r0 - 1, c0, c1)) if a.dtype == np.float32
         else (S(r0, r1, 0, c1) + S(0, r0 - 1, c0, c1)) % (1 << 32),
-        "GSAT": [[S(0, r0 + i, 0, c0 + j) for j in range(c1 - c0 + 1)] for i in range(r1 - r0 + 1)],
+        "GSAT": [[S(0, r0 + i, 0, c0 + j) for j in range(c1 - c0 + 1)] for i in range(r1 - r0 + 1)]
+        if with_gsat else None,
     }
     return out
 

@@ -23,7 +23,8 @@ _lib.lib()  # load now: fail loudly at import if the native library is missing
 __all__ = [
     "sat", "sat_batched", "sat_batched_u8", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
     "strip_layout", "broadcast_unique_id",
-    "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "release_workspaces",
+    "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "debug_workspace",
+    "release_stream_workspace", "release_workspaces",
     "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
 ]
 
@@ -47,6 +48,12 @@ def _stream_ptr(stream) -> int:
     torch = _torch()
     s = torch.cuda.current_stream() if stream is None else stream
     return int(s.cuda_stream)
+
+
+def _check_vec_out(out, n: int, dtype, device, name: str = "out"):
+    """A caller-supplied output vector: contiguous, `n` elements of `dtype` on `device`."""
+    if out.dtype != dtype or out.numel() != n or not out.is_contiguous() or out.device != device:
+        raise ValueError(f"{name} must be a contiguous tensor of {n} elements, dtype {dtype}, on {device}")
 
 
 def _matrix(t, name: str):
@@ -193,6 +200,7 @@ def rect_sums(b, rects, out=None, *, stream=None):
     n = rects.shape[0]
     if out is None:
         out = torch.empty(n, dtype=b.dtype, device=b.device)
+    _check_vec_out(out, n, b.dtype, b.device)
     with torch.cuda.device(b.device):
         check(_lib.lib().sat_rect_sums(_dtype_code(b), b.data_ptr(), rows, cols, pitch, rects.data_ptr(), n,
                                        out.data_ptr(), _stream_ptr(stream)), "sat_rect_sums")
@@ -205,6 +213,7 @@ def strip_colsum(src, out=None, *, stream=None):
     rows, cols, pitch = _matrix(src, "src")
     if out is None:
         out = torch.empty(cols, dtype=src.dtype, device=src.device)
+    _check_vec_out(out, cols, src.dtype, src.device)
     with torch.cuda.device(src.device):
         check(_lib.lib().sat_strip_colsum(_dtype_code(src), src.data_ptr(), out.data_ptr(), rows, cols, pitch,
                                           _stream_ptr(stream)), "sat_strip_colsum")
@@ -214,11 +223,12 @@ def strip_colsum(src, out=None, *, stream=None):
 def carry_prefix(gathered, rank: int, out=None, *, stream=None):
     """Carry row of ``rank`` from the (nranks x cols) gathered column sums (device)."""
     torch = _torch()
-    if gathered.dim() != 2 or not gathered.is_contiguous():
-        raise ValueError("gathered must be a contiguous (nranks, cols) tensor")
+    if gathered.dim() != 2 or not gathered.is_contiguous() or not gathered.is_cuda:
+        raise ValueError("gathered must be a contiguous (nranks, cols) CUDA tensor")
     nranks, cols = gathered.shape
     if out is None:
         out = torch.empty(cols, dtype=gathered.dtype, device=gathered.device)
+    _check_vec_out(out, cols, gathered.dtype, gathered.device)
     with torch.cuda.device(gathered.device):
         check(_lib.lib().sat_carry_prefix(_dtype_code(gathered), gathered.data_ptr(), nranks, rank, cols,
                                           out.data_ptr(), _stream_ptr(stream)), "sat_carry_prefix")
@@ -307,6 +317,9 @@ def sat_sharded(strip, out=None, *, comm: Comm, stream=None, check_layout: bool 
         strip_layout(rows, cols, _dtype_code(strip), comm.group)
     if out is None:
         out = torch.empty_strided((rows, cols), (pitch, 1), dtype=strip.dtype, device=strip.device)
+    if out.dtype != strip.dtype or out.device != strip.device or tuple(out.shape) != (rows, cols) or \
+            (rows > 0 and _matrix(out, "out")[2] != pitch):
+        raise ValueError("out must match strip in shape, row stride, dtype and device")
     with torch.cuda.device(strip.device):
         check(_lib.lib().sat_compute_sharded(comm._h, _dtype_code(strip), strip.data_ptr(), out.data_ptr(), rows,
                                              cols, pitch, _stream_ptr(stream)), "sat_compute_sharded")
@@ -348,6 +361,27 @@ def debug_tile_order(R: int, C: int, order: int = 0, device=None):
     with torch.cuda.device(out.device):
         check(_lib.lib().sat_debug_tile_order(R, C, order, out.data_ptr(), _stream_ptr(None)), "sat_debug_tile_order")
     return out
+
+
+def debug_workspace(stream=None, words: bool = True):
+    """Test hook (sat_debug_workspace): the published aggregate words of the last sat_compute launch on
+    ``stream`` (current stream by default).  Returns (info dict, numpy uint64 array or None): row slots
+    [R*C][tile_rows], column slots [R*C][tile_cols], corner slots [R*C]."""
+    import numpy as np
+
+    info = _lib.SatWsInfo()
+    sp = _stream_ptr(stream)
+    check(_lib.lib().sat_debug_workspace(sp, None, 0, ctypes.byref(info)), "sat_debug_workspace")
+    d = {f: getattr(info, f) for f, _ in _lib.SatWsInfo._fields_}
+    if not words:
+        return d, None
+    buf = np.empty(max(1, d["words"]), dtype=np.uint64)
+    check(_lib.lib().sat_debug_workspace(sp, buf.ctypes.data, buf.size, ctypes.byref(info)), "sat_debug_workspace")
+    return d, buf[: d["words"]]
+
+
+def release_stream_workspace(stream=None) -> None:
+    check(_lib.lib().sat_release_stream_workspace(_stream_ptr(stream)), "sat_release_stream_workspace")
 
 
 def release_workspaces() -> None:

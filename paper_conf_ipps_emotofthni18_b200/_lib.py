@@ -26,7 +26,7 @@ EXPORTS = (
     "sat_strip_colsum",
     "sat_carry_prefix", "sat_comm_get_unique_id", "sat_comm_init", "sat_comm_destroy", "sat_compute_sharded",
     "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order", "sat_debug_stats", "sat_debug_trace",
-    "sat_release_workspaces", "sat_status_string", "sat_last_error_detail", "sat_version",
+    "sat_debug_workspace", "sat_release_stream_workspace", "sat_release_workspaces", "sat_status_string", "sat_last_error_detail", "sat_version",
 )
 
 
@@ -37,6 +37,11 @@ class SatPlan(ctypes.Structure):
         ("variant", ctypes.c_int32), ("order", ctypes.c_int32), ("family", ctypes.c_int32),
         ("reserved", ctypes.c_int32),
     ]
+
+
+class SatWsInfo(ctypes.Structure):
+    _fields_ = [("tile_rows", ctypes.c_int32), ("tile_cols", ctypes.c_int32), ("R", ctypes.c_int32),
+                ("C", ctypes.c_int32), ("words", ctypes.c_int64)]
 
 
 class SatError(RuntimeError):
@@ -73,6 +78,8 @@ def _declare(lib):
         "sat_debug_tile_order": [_i64, _i64, _int, _vp, _vp],
         "sat_debug_stats": [_vp, _int, ctypes.POINTER(_int), ctypes.POINTER(_int)],
         "sat_debug_trace": [_vp, _i64, ctypes.POINTER(_i64)],
+        "sat_debug_workspace": [_vp, _vp, _i64, ctypes.POINTER(SatWsInfo)],
+        "sat_release_stream_workspace": [_vp],
         "sat_release_workspaces": [],
         "sat_status_string": [_int],
         "sat_last_error_detail": [],

@@ -283,6 +283,15 @@ sat_status_t device_info(int dev, DeviceInfo** out) {
     return SAT_OK;
 }
 
+// SM count of `dev` (cached; takes g_mu)
+sat_status_t device_sms(int dev, int* sms) {
+    std::lock_guard<std::mutex> lk(g_mu);
+    DeviceInfo* di;
+    sat_status_t s = device_info(dev, &di);
+    if (s == SAT_OK) *sms = di->sms;
+    return s;
+}
+
 sat_status_t occupancy(int dev, int vi, int dt, bool tma, bool carry, int* occ) {
     DeviceInfo* di;
     sat_status_t s = device_info(dev, &di);
@@ -309,6 +318,7 @@ sat_status_t occupancy(int dev, int vi, int dt, bool tma, bool carry, int* occ) 
 struct Workspace {
     int dev = 0;
     cudaStream_t stream = nullptr;
+    std::mutex mu;  // growth + launch on this (device, stream); g_mu only guards the map
     Ctrl* ctrl = nullptr;
     uint64_t* slots = nullptr;
     size_t slot_words = 0;
@@ -319,6 +329,7 @@ struct Workspace {
     int64_t trace_tiles = 0;
     void* scratch = nullptr;  // colsum partials etc.
     size_t scratch_bytes = 0;
+    int last_TR = 0, last_TC = 0, last_R = 0, last_C = 0;  // tile grid of the last launch (sat_debug_workspace)
 };
 std::map<std::pair<int, cudaStream_t>, Workspace*> g_ws;
 Workspace* g_last_stats = nullptr;
@@ -326,66 +337,73 @@ Workspace* g_last_stats = nullptr;
 sat_status_t reset_ctrl(Workspace* w) {
     Ctrl init{0u, 0u, 1u, 0u};
     SAT_CUDA(cudaMemcpyAsync(w->ctrl, &init, sizeof(Ctrl), cudaMemcpyHostToDevice, w->stream));
-    SAT_CUDA(cudaStreamSynchronize(w->stream));
+    SAT_CUDA(cudaStreamSynchronize(w->stream));  // `init` lives on this stack frame
     return SAT_OK;
 }
 
-sat_status_t get_workspace(int dev, cudaStream_t st, size_t slot_words, Workspace** out) {
+// The workspace of (dev, st), created on first use (one synchronising control-block reset).  The
+// caller locks w->mu before growing it (grow_slots) or launching with it.
+sat_status_t find_workspace(int dev, cudaStream_t st, Workspace** out) {
+    std::lock_guard<std::mutex> lk(g_mu);
     auto key = std::make_pair(dev, st);
     auto it = g_ws.find(key);
-    Workspace* w;
-    if (it == g_ws.end()) {
-        w = new Workspace();
-        w->dev = dev;
-        w->stream = st;
-        cudaError_t e = cudaMalloc(&w->ctrl, 256);
-        if (e != cudaSuccess) {
-            delete w;
-            return fail(SAT_ERR_OUT_OF_MEMORY, "workspace control block: %s", cudaGetErrorString(e));
-        }
-        sat_status_t s = reset_ctrl(w);
-        if (s != SAT_OK) {
-            cudaFree(w->ctrl);
-            delete w;
-            return s;
-        }
-        g_ws[key] = w;
-    } else {
-        w = it->second;
+    if (it != g_ws.end()) {
+        *out = it->second;
+        return SAT_OK;
     }
+    Workspace* w = new Workspace();
+    w->dev = dev;
+    w->stream = st;
+    cudaError_t e = cudaMalloc(&w->ctrl, 256);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        delete w;
+        return fail(SAT_ERR_OUT_OF_MEMORY, "workspace control block: %s", cudaGetErrorString(e));
+    }
+    sat_status_t s = reset_ctrl(w);
+    if (s != SAT_OK) {
+        cudaFree(w->ctrl);
+        delete w;
+        return s;
+    }
+    g_ws[key] = w;
+    *out = w;
+    return SAT_OK;
+}
+
+// Grow the status-word slots to >= slot_words (stream-ordered: cudaFreeAsync / cudaMallocAsync /
+// cudaMemsetAsync on the workspace's stream, no host synchronisation).  New words are zeroed: epoch 0
+// never matches a launch epoch (>= 1), so they read "not published".
+sat_status_t grow_slots(Workspace* w, size_t slot_words) {
     if (slot_words > w->slot_words) {
-        size_t want = slot_words + slot_words / 4;
-        SAT_CUDA(cudaStreamSynchronize(st));
-        if (w->slots) SAT_CUDA(cudaFree(w->slots));
+        const size_t want = slot_words + slot_words / 4;
+        if (w->slots) SAT_CUDA(cudaFreeAsync(w->slots, w->stream));
         w->slots = nullptr;
         w->slot_words = 0;
-        cudaError_t e = cudaMalloc(&w->slots, want * sizeof(uint64_t));
+        cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&w->slots), want * sizeof(uint64_t), w->stream);
         if (e != cudaSuccess) {
             cudaGetLastError();
             return fail(SAT_ERR_OUT_OF_MEMORY, "workspace slots (%zu bytes): %s", want * 8, cudaGetErrorString(e));
         }
-        SAT_CUDA(cudaMemsetAsync(w->slots, 0, want * sizeof(uint64_t), st));
+        SAT_CUDA(cudaMemsetAsync(w->slots, 0, want * sizeof(uint64_t), w->stream));
         w->slot_words = want;
     }
     // Epoch wrap (after ~2^30 launches on this workspace): clear the slots and restart at epoch 1.
     if (w->calls + 2 >= sat::kEpochMax) {
-        SAT_CUDA(cudaStreamSynchronize(st));
-        SAT_CUDA(cudaMemsetAsync(w->slots, 0, w->slot_words * sizeof(uint64_t), st));
+        SAT_CUDA(cudaMemsetAsync(w->slots, 0, w->slot_words * sizeof(uint64_t), w->stream));
         sat_status_t s = reset_ctrl(w);
         if (s != SAT_OK) return s;
         w->calls = 0;
     }
-    *out = w;
     return SAT_OK;
 }
 
 sat_status_t get_scratch(Workspace* w, size_t bytes, void** out) {
     if (bytes > w->scratch_bytes) {
-        SAT_CUDA(cudaStreamSynchronize(w->stream));
-        if (w->scratch) SAT_CUDA(cudaFree(w->scratch));
+        if (w->scratch) SAT_CUDA(cudaFreeAsync(w->scratch, w->stream));
         w->scratch = nullptr;
         w->scratch_bytes = 0;
-        cudaError_t e = cudaMalloc(&w->scratch, bytes);
+        cudaError_t e = cudaMallocAsync(&w->scratch, bytes, w->stream);
         if (e != cudaSuccess) {
             cudaGetLastError();
             return fail(SAT_ERR_OUT_OF_MEMORY, "scratch (%zu bytes): %s", bytes, cudaGetErrorString(e));
@@ -394,6 +412,19 @@ sat_status_t get_scratch(Workspace* w, size_t bytes, void** out) {
     }
     *out = w->scratch;
     return SAT_OK;
+}
+
+// Synchronises the workspace's stream and frees its buffers (the caller has removed it from g_ws).
+void free_workspace(Workspace* w) {
+    {
+        std::lock_guard<std::mutex> wlk(w->mu);
+        cudaStreamSynchronize(w->stream);
+        if (w->slots) cudaFree(w->slots);
+        if (w->scratch) cudaFree(w->scratch);
+        if (w->ctrl) cudaFree(w->ctrl);
+        if (w->stats) cudaFree(w->stats);
+    }
+    delete w;
 }
 
 // ------------------------------------------------------------------ TMA tensor maps
@@ -524,19 +555,26 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
 
     int dev = 0;
     SAT_CUDA(cudaGetDevice(&dev));
-    std::lock_guard<std::mutex> lk(g_mu);
-    int occ = 0;
-    if ((s = occupancy(dev, pl.vi, dt, pl.tma, carry != nullptr, &occ)) != SAT_OK) return s;
-    DeviceInfo* di;
-    if ((s = device_info(dev, &di)) != SAT_OK) return s;
-    int per_sm = (g_ctas_per_sm > 0 && g_ctas_per_sm < occ) ? g_ctas_per_sm : occ;
-    int64_t grid = static_cast<int64_t>(di->sms) * per_sm;
-    if (g_max_ctas > 0 && grid > g_max_ctas) grid = g_max_ctas;
+    int occ = 0, sms = 0, max_ctas = 0, ctas_per_sm = 0;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        if ((s = occupancy(dev, pl.vi, dt, pl.tma, carry != nullptr, &occ)) != SAT_OK) return s;
+        DeviceInfo* di;
+        if ((s = device_info(dev, &di)) != SAT_OK) return s;
+        sms = di->sms;
+        max_ctas = g_max_ctas;
+        ctas_per_sm = g_ctas_per_sm;
+    }
+    int per_sm = (ctas_per_sm > 0 && ctas_per_sm < occ) ? ctas_per_sm : occ;
+    int64_t grid = static_cast<int64_t>(sms) * per_sm;
+    if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
     if (grid > pl.ntiles) grid = pl.ntiles;
 
     Workspace* w;
+    if ((s = find_workspace(dev, st, &w)) != SAT_OK) return s;
+    std::lock_guard<std::mutex> wlk(w->mu);
     const size_t words = static_cast<size_t>(pl.ntiles) * (v.TR + v.TC + 1);
-    if ((s = get_workspace(dev, st, words, &w)) != SAT_OK) return s;
+    if ((s = grow_slots(w, words)) != SAT_OK) return s;
 
     CUtensorMap mi, mo;
     std::memset(&mi, 0, sizeof(mi));
@@ -575,6 +613,7 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
     if (u8) p.src = nullptr;
 #if SAT_STATS
     {
+        std::lock_guard<std::mutex> lk(g_mu);
         const size_t need = static_cast<size_t>(grid) * sat::kNumStats + 8 * static_cast<size_t>(pl.ntiles);
         if (w->stats_words < need) {
             if (w->stats) cudaFree(w->stats);
@@ -586,12 +625,16 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
         SAT_CUDA(cudaMemsetAsync(w->stats, 0, need * 8, st));
         p.stats = w->stats;
         p.trace = w->stats + static_cast<size_t>(grid) * sat::kNumStats;
+        g_last_stats = w;
     }
-    g_last_stats = w;
 #endif
     cudaError_t e = v.launch[dt](pl.tma, carry != nullptr, dim3(static_cast<unsigned>(grid)), st, mi, mo, &p);
-    if (e != cudaSuccess) return cuda_fail(e, "sat_tiles_kernel launch");
+    if (e != cudaSuccess) return cuda_fail(e, "SAT kernel launch");
     w->calls++;
+    w->last_TR = v.TR;
+    w->last_TC = v.TC;
+    w->last_R = pl.R;
+    w->last_C = pl.C;
     return SAT_OK;
 }
 
@@ -609,14 +652,13 @@ sat_status_t colsum_impl(sat_dtype_t dt, const void* src, void* colsum, int64_t 
     }
     int dev = 0;
     SAT_CUDA(cudaGetDevice(&dev));
-    std::lock_guard<std::mutex> lk(g_mu);
-    DeviceInfo* di;
-    sat_status_t s = device_info(dev, &di);
+    int sms = 0;
+    sat_status_t s = device_sms(dev, &sms);
     if (s != SAT_OK) return s;
     const bool vec = ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) && (pitch % 4 == 0);
     const int64_t bx = (cols + (vec ? 1023 : 255)) / (vec ? 1024 : 256);
     // one full wave: at most 8 blocks of 256 threads per SM (a partial second wave doubles the time)
-    int64_t nseg = (static_cast<int64_t>(di->sms) * 8) / bx;
+    int64_t nseg = (static_cast<int64_t>(sms) * 8) / bx;
     const int64_t max_seg = (rows + 7) / 8;
     if (nseg > max_seg) nseg = max_seg;
     if (nseg > 65535) nseg = 65535;
@@ -624,7 +666,8 @@ sat_status_t colsum_impl(sat_dtype_t dt, const void* src, void* colsum, int64_t 
     const int64_t seg = (rows + nseg - 1) / nseg;
     nseg = (rows + seg - 1) / seg;
     Workspace* w;
-    if ((s = get_workspace(dev, st, 0, &w)) != SAT_OK) return s;
+    if ((s = find_workspace(dev, st, &w)) != SAT_OK) return s;
+    std::lock_guard<std::mutex> wlk(w->mu);
     void* partial;
     if ((s = get_scratch(w, static_cast<size_t>(nseg * cols) * 4, &partial)) != SAT_OK) return s;
     dim3 g1(static_cast<unsigned>(bx), static_cast<unsigned>(nseg));
@@ -680,7 +723,7 @@ sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, in
     int dev = 0;
     SAT_CUDA(cudaGetDevice(&dev));
     int sms = 0;
-    SAT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    if ((s = device_sms(dev, &sms)) != SAT_OK) return s;
     const int64_t gx = (cols + 1023) / 1024;
     int64_t gy = (static_cast<int64_t>(sms) * 8 + gx - 1) / gx;
     if (gy > rows) gy = rows;
@@ -777,7 +820,8 @@ int batch_nwr(int64_t cols) { return cols <= 128 ? 1 : cols <= 256 ? 2 : cols <=
 sat_status_t batch_grid(int64_t batch, int nwr, unsigned* grid) {
     int dev = 0, sms = 0;
     SAT_CUDA(cudaGetDevice(&dev));
-    SAT_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    sat_status_t s = device_sms(dev, &sms);
+    if (s != SAT_OK) return s;
     const int64_t cap = static_cast<int64_t>(sms) * 64;  // resident blocks are far fewer; the rest queue
     const int64_t ctas = nwr == 1 ? (batch + 3) / 4 : batch;  // one-warp CTAs hold 4 matrices (kBatchIpb)
     *grid = static_cast<unsigned>(ctas < cap ? ctas : cap);
@@ -843,12 +887,18 @@ sat_status_t batched_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ba
 }
 
 // ------------------------------------------------------------------ end-to-end host pipeline
+// One staging buffer, copy-stream pair and event set per device.  `mu` is held for a whole
+// sat_compute_host call (through its final synchronisations), so concurrent calls on one device
+// run one after the other instead of sharing the buffer.
+constexpr int kHostMaxStrips = 16;
 struct Staging {
+    std::mutex mu;
     void* buf = nullptr;
     size_t bytes = 0;
     cudaStream_t h2d = nullptr, d2h = nullptr;
+    cudaEvent_t ev[2 * kHostMaxStrips] = {};
 };
-std::map<int, Staging> g_staging;
+std::map<int, Staging*> g_staging;
 
 // ------------------------------------------------------------------ NCCL (dlopen)
 #if defined(SAT_HAVE_NCCL_H)
@@ -959,34 +1009,37 @@ SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, v
     Staging* sg;
     {
         std::lock_guard<std::mutex> lk(g_mu);
-        sg = &g_staging[dev];
-        const size_t bytes = static_cast<size_t>(rows) * pitch * 4;
-        if (!sg->h2d) {
-            SAT_CUDA(cudaStreamCreateWithFlags(&sg->h2d, cudaStreamNonBlocking));
-            SAT_CUDA(cudaStreamCreateWithFlags(&sg->d2h, cudaStreamNonBlocking));
-        }
-        if (bytes > sg->bytes) {
-            if (sg->buf) SAT_CUDA(cudaFree(sg->buf));
-            sg->buf = nullptr;
-            sg->bytes = 0;
-            cudaError_t e = cudaMalloc(&sg->buf, bytes);
-            if (e != cudaSuccess) {
-                cudaGetLastError();
-                return fail(SAT_ERR_OUT_OF_MEMORY, "staging buffer (%zu bytes)", bytes);
-            }
-            sg->bytes = bytes;
-        }
+        auto it = g_staging.find(dev);
+        if (it == g_staging.end()) it = g_staging.emplace(dev, new Staging()).first;
+        sg = it->second;
     }
-    // strips of >= 2 MiB, at most 16, multiples of 128 rows
+    std::lock_guard<std::mutex> slk(sg->mu);
+    const size_t bytes = static_cast<size_t>(rows) * pitch * 4;
+    if (!sg->h2d) {
+        SAT_CUDA(cudaStreamCreateWithFlags(&sg->h2d, cudaStreamNonBlocking));
+        SAT_CUDA(cudaStreamCreateWithFlags(&sg->d2h, cudaStreamNonBlocking));
+        for (auto& e : sg->ev) SAT_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
+    if (bytes > sg->bytes) {
+        // the previous call synchronised all three streams before releasing sg->mu
+        if (sg->buf) SAT_CUDA(cudaFree(sg->buf));
+        sg->buf = nullptr;
+        sg->bytes = 0;
+        cudaError_t e = cudaMalloc(&sg->buf, bytes);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(SAT_ERR_OUT_OF_MEMORY, "staging buffer (%zu bytes)", bytes);
+        }
+        sg->bytes = bytes;
+    }
+    // strips of >= 2 MiB, at most kHostMaxStrips, multiples of 128 rows
     const int64_t row_bytes = pitch * 4;
     int64_t nstrips = (rows * row_bytes) / (int64_t(2) << 20);
     if (nstrips < 1) nstrips = 1;
-    if (nstrips > 16) nstrips = 16;
+    if (nstrips > kHostMaxStrips) nstrips = kHostMaxStrips;
     int64_t h = (rows + nstrips - 1) / nstrips;
     h = ((h + 127) / 128) * 128;
     nstrips = (rows + h - 1) / h;
-    std::vector<cudaEvent_t> ev(2 * nstrips);
-    for (auto& e : ev) SAT_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     sat_status_t status = SAT_OK;
     char* dbuf = static_cast<char*>(sg->buf);
     for (int64_t k = 0; k < nstrips && status == SAT_OK; ++k) {
@@ -997,8 +1050,8 @@ SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, v
         char* hd = static_cast<char*>(host_dst) + r0 * row_bytes;
         cudaError_t e = cudaMemcpy2DAsync(dstrip, row_bytes, hs, row_bytes, cols * 4, nr, cudaMemcpyHostToDevice,
                                           sg->h2d);
-        if (e == cudaSuccess) e = cudaEventRecord(ev[2 * k], sg->h2d);
-        if (e == cudaSuccess) e = cudaStreamWaitEvent(st, ev[2 * k], 0);
+        if (e == cudaSuccess) e = cudaEventRecord(sg->ev[2 * k], sg->h2d);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(st, sg->ev[2 * k], 0);
         if (e != cudaSuccess) {
             status = cuda_fail(e, "host pipeline H2D");
             break;
@@ -1006,8 +1059,8 @@ SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, v
         const void* carry = (k > 0) ? static_cast<const void*>(dstrip - row_bytes) : nullptr;
         status = compute_impl(dtype, dstrip, dstrip, nr, cols, pitch, carry, st);
         if (status != SAT_OK) break;
-        e = cudaEventRecord(ev[2 * k + 1], st);
-        if (e == cudaSuccess) e = cudaStreamWaitEvent(sg->d2h, ev[2 * k + 1], 0);
+        e = cudaEventRecord(sg->ev[2 * k + 1], st);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(sg->d2h, sg->ev[2 * k + 1], 0);
         if (e == cudaSuccess)
             e = cudaMemcpy2DAsync(hd, row_bytes, dstrip, row_bytes, cols * 4, nr, cudaMemcpyDeviceToHost, sg->d2h);
         if (e != cudaSuccess) status = cuda_fail(e, "host pipeline D2H");
@@ -1015,7 +1068,6 @@ SAT_API sat_status_t sat_compute_host(sat_dtype_t dtype, const void* host_src, v
     cudaError_t e1 = cudaStreamSynchronize(sg->d2h);
     cudaError_t e2 = cudaStreamSynchronize(st);
     cudaError_t e3 = cudaStreamSynchronize(sg->h2d);
-    for (auto& e : ev) cudaEventDestroy(e);
     if (status != SAT_OK) return status;
     if (e1 != cudaSuccess) return cuda_fail(e1, "host pipeline sync");
     if (e2 != cudaSuccess) return cuda_fail(e2, "host pipeline sync");
@@ -1079,7 +1131,7 @@ SAT_API sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, con
 #if defined(SAT_HAVE_NCCL_H)
     if (!comm) return fail(SAT_ERR_INVALID_VALUE, "null comm");
     if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype");
-    if (strip_rows < 0 || cols <= 0 || pitch < cols) return fail(SAT_ERR_INVALID_VALUE, "bad sizes");
+    if (cols <= 0) return fail(SAT_ERR_INVALID_VALUE, "bad sizes");  // cols, dtype, comm: equal on all ranks
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const size_t need = static_cast<size_t>(cols) * 4 * (comm->nranks + 2);
     if (need > comm->bytes) {
@@ -1097,11 +1149,26 @@ SAT_API sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, con
     void* colsum = base;
     void* gathered = base + cols * 4;
     void* carry = base + cols * 4 * (comm->nranks + 1);
-    sat_status_t s = colsum_impl(dtype, strip_src, colsum, strip_rows, cols, pitch, st);
-    if (s != SAT_OK) return s;
+    // Every rank-local check runs before the collective.  A rank whose arguments or column-sum launch
+    // fail still joins the all-gather (with a zero vector) so that no other rank blocks in it, then
+    // returns its own error.
+    sat_status_t local = (strip_rows < 0 || pitch < cols)
+                             ? fail(SAT_ERR_INVALID_VALUE, "bad sizes strip_rows=%lld pitch=%lld", (long long)strip_rows,
+                                    (long long)pitch)
+                             : (strip_rows > 0 ? validate(strip_src, strip_dst, strip_rows, cols, pitch) : SAT_OK);
+    if (local == SAT_OK) local = colsum_impl(dtype, strip_src, colsum, strip_rows, cols, pitch, st);
+    if (local != SAT_OK) {
+        const std::string detail = g_detail;
+        cudaMemsetAsync(colsum, 0, cols * 4, st);
+        g_nccl.allGather(colsum, gathered, static_cast<size_t>(cols), dtype == SAT_INT32 ? ncclUint32 : ncclFloat32,
+                         comm->comm, st);
+        g_detail = detail;
+        return local;
+    }
     ncclResult_t r = g_nccl.allGather(colsum, gathered, static_cast<size_t>(cols),
                                       dtype == SAT_INT32 ? ncclUint32 : ncclFloat32, comm->comm, st);
     if (r != ncclSuccess) return nccl_fail(r, "ncclAllGather");
+    sat_status_t s;
     if ((s = carry_impl(dtype, gathered, comm->nranks, comm->rank, cols, carry, st)) != SAT_OK) return s;
     if (strip_rows == 0) return SAT_OK;
     return compute_impl(dtype, strip_src, strip_dst, strip_rows, cols, pitch, carry, st);
@@ -1226,27 +1293,74 @@ SAT_API sat_status_t sat_debug_trace(int64_t* out, int64_t max_tiles, int64_t* n
 #endif
 }
 
+SAT_API sat_status_t sat_release_stream_workspace(void* stream) {
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    Workspace* w = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        auto it = g_ws.find(std::make_pair(dev, static_cast<cudaStream_t>(stream)));
+        if (it == g_ws.end()) return SAT_OK;
+        w = it->second;
+        g_ws.erase(it);
+        if (g_last_stats == w) g_last_stats = nullptr;
+    }
+    free_workspace(w);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "release");
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_debug_workspace(void* stream, uint64_t* host_out, int64_t max_words, sat_ws_info_t* info) {
+    if (!info) return fail(SAT_ERR_INVALID_VALUE, "null info");
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    Workspace* w = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        auto it = g_ws.find(std::make_pair(dev, static_cast<cudaStream_t>(stream)));
+        if (it == g_ws.end()) return fail(SAT_ERR_INVALID_VALUE, "no workspace for this (device, stream)");
+        w = it->second;
+    }
+    std::lock_guard<std::mutex> wlk(w->mu);
+    const int64_t tiles = static_cast<int64_t>(w->last_R) * w->last_C;
+    info->tile_rows = w->last_TR;
+    info->tile_cols = w->last_TC;
+    info->R = w->last_R;
+    info->C = w->last_C;
+    info->words = tiles * (w->last_TR + w->last_TC + 1);
+    if (!host_out) return SAT_OK;
+    if (max_words < info->words) return fail(SAT_ERR_INVALID_VALUE, "host_out holds %lld < %lld words",
+                                             (long long)max_words, (long long)info->words);
+    SAT_CUDA(cudaStreamSynchronize(w->stream));
+    if (info->words > 0)
+        SAT_CUDA(cudaMemcpy(host_out, w->slots, static_cast<size_t>(info->words) * 8, cudaMemcpyDeviceToHost));
+    return SAT_OK;
+}
+
 SAT_API sat_status_t sat_release_workspaces(void) {
     std::lock_guard<std::mutex> lk(g_mu);
     int cur = 0;
     cudaGetDevice(&cur);
     for (auto& kv : g_ws) {
-        Workspace* w = kv.second;
-        cudaSetDevice(w->dev);
-        cudaStreamSynchronize(w->stream);
-        if (w->slots) cudaFree(w->slots);
-        if (w->scratch) cudaFree(w->scratch);
-        if (w->ctrl) cudaFree(w->ctrl);
-        if (w->stats) cudaFree(w->stats);
-        delete w;
+        cudaSetDevice(kv.second->dev);
+        free_workspace(kv.second);
     }
     g_ws.clear();
     g_last_stats = nullptr;
     for (auto& kv : g_staging) {
         cudaSetDevice(kv.first);
-        if (kv.second.buf) cudaFree(kv.second.buf);
-        if (kv.second.h2d) cudaStreamDestroy(kv.second.h2d);
-        if (kv.second.d2h) cudaStreamDestroy(kv.second.d2h);
+        Staging* sg = kv.second;
+        {
+            std::lock_guard<std::mutex> slk(sg->mu);
+            if (sg->buf) cudaFree(sg->buf);
+            if (sg->h2d) {
+                cudaStreamDestroy(sg->h2d);
+                cudaStreamDestroy(sg->d2h);
+                for (auto& e : sg->ev) cudaEventDestroy(e);
+            }
+        }
+        delete sg;
     }
     g_staging.clear();
     cudaSetDevice(cur);
