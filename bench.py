@@ -251,6 +251,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--sweep", action="store_true")
     ap.add_argument("--no-extras", action="store_true", help="skip the other BASELINE configs (4K^2, sweep, 64K^2)")
+    ap.add_argument("--sharded", choices=["chain", "gather"], default="chain",
+                    help="N>1: chained strips in one pass (default) or column sums + NCCL all-gather + SAT")
     ap.add_argument("--variant", type=int, default=-1)
     ap.add_argument("--order", type=int, default=0)
     ap.add_argument("--ctas-per-sm", type=int, default=0)
@@ -292,13 +294,19 @@ def main():
     satgen.fill_tensor(x, 1447, dist_name, row0=row0)
     x = x.view(tdt)
     y = torch.empty_like(x)
-    comm = sat.Comm() if world > 1 else None
+    comm = chain = None
+    if world > 1 and args.sharded == "gather":
+        comm = sat.Comm()
+    elif world > 1:
+        chain = sat.Chain(cols)
 
     def step():
-        if comm is None:
-            sat.sat(x, out=y)
-        else:
+        if comm is not None:
             sat.sat_sharded(x, out=y, comm=comm)
+        elif chain is not None:
+            sat.sat_chained(x, out=y, chain=chain)
+        else:
+            sat.sat(x, out=y)
 
     def barrier():
         if world > 1:
@@ -342,7 +350,7 @@ def main():
     m1.record(stream)
     torch.cuda.synchronize()
     memcpy_ms = m0.elapsed_time(m1) / args.steps
-    sat.sat(x, out=y) if comm is None else sat.sat_sharded(x, out=y, comm=comm)
+    step()
     torch.cuda.synchronize()
 
     # ---- end to end through the C ABI with host buffers (rank 0 of N=1 only; PCIe-bound)
@@ -369,7 +377,8 @@ def main():
                        "tile": [plan["tile_rows"], plan["tile_cols"]], "ctas": plan["ctas"],
                        "variant": plan["variant"], "order": order_name(plan["order"]),
                        "l2": "inputs (4 B x n^2) larger than the 126 MB L2; no flush",
-                       "parallelism": "single GPU" if world == 1 else f"strips x{world}"},
+                       "parallelism": "single GPU" if world == 1 else
+                       f"strips x{world} ({'sat_compute_chained' if chain is not None else 'sat_compute_sharded'})"},
             "hbm_gbs": achieved,
             "memcpy": {"ms": memcpy_ms, "gbs": nrows * cols * BYTES_PER_ELEM / (memcpy_ms / 1e3) / 1e9,
                        "overhead_pct": (ms - memcpy_ms) / memcpy_ms * 100.0, "ratio": ms / memcpy_ms,
@@ -380,7 +389,7 @@ def main():
                          "kernel": {2: "sat_tm_kernel"}.get(plan["family"], "sat_tiles_kernel"),
                          "bytes_per_elem": BYTES_PER_ELEM,
                          "timing": "CUDA events on the launching stream around the K timed launches"},
-            "gpu_launches": args.steps * (1 if world == 1 else 4),
+            "gpu_launches": args.steps * (4 if comm is not None else 1),
             "clocks": clk,
             "e2e": e2e,
         }
@@ -392,6 +401,9 @@ def main():
         print(json.dumps(line), flush=True)
     if comm is not None:
         comm.close()
+    if chain is not None:
+        chain.close()
+    if world > 1:
         dist.destroy_process_group()
     return 0
 
@@ -544,7 +556,71 @@ def run_extras(args, sat, satgen, torch, x, peak) -> dict:
     out["i32_64k_single_gpu"] = {"rows": n, "cols": n, "sat_ms": t_sat, "memcpy_ms": t_cp,
                                  "overhead_pct": (t_sat - t_cp) / t_cp * 100.0, "gbs": gbs, "frac": gbs / peak,
                                  "note": "in place; 5 launches between CUDA events"}
+    out["chain_64k"] = chain_projection(torch, sat, satgen, n, t_sat)
     return out
+
+
+def chain_projection(torch, sat, satgen, n, single_ms) -> dict:
+    """configs[4] (64K^2 int32 strips on N GPUs) with the chained partition, emulated on this one GPU:
+    * per_rank_ms: every rank's kernel alone on the whole GPU, ranks one after the other on one stream
+      (each finds its upstream column sums already in its inbox): the per-GPU work of an N-GPU run;
+      projected efficiency = single-pass 64K^2 time / (N * slowest rank), i.e. linear scaling minus the
+      per-rank overheads (the start-up lag of one tile column and NVLink latency are not in it);
+    * concurrent_ms: all N ranks' kernels at once on N streams, the GPU's SMs split N ways, the whole
+      in-kernel protocol (pushes, inbox waits, back-pressure) running; efficiency = single / concurrent.
+    In place on one 16 GiB matrix (timings do not depend on the values)."""
+    res = {"single_pass_ms": single_ms}
+    x = torch.empty((n, n), dtype=torch.int32, device="cuda")
+    satgen.fill_tensor(x, 1447, "u32")
+    sms = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+    for N in (2, 4, 8):
+        h = n // N
+        parts = [x[r * h:(r + 1) * h] for r in range(N)]
+        chains = sat.Chain.local(N, n)
+        try:
+            per = [0.0] * N
+            for it in range(4):
+                evs = [torch.cuda.Event(enable_timing=True) for _ in range(N + 1)]
+                evs[0].record()
+                for r in range(N):
+                    sat.sat_chained(parts[r], out=parts[r], chain=chains[r])
+                    evs[r + 1].record()
+                torch.cuda.synchronize()
+                if it > 0:
+                    per = [max(per[r], evs[r].elapsed_time(evs[r + 1])) if it > 1 else evs[r].elapsed_time(evs[r + 1])
+                           for r in range(N)]
+            streams = [torch.cuda.Stream() for _ in range(N)]
+            sat.set_max_ctas(sms // N)
+            try:
+                times = []
+                for it in range(4):
+                    torch.cuda.synchronize()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record()
+                    for st in streams:
+                        st.wait_event(e0)
+                    for r in range(N):
+                        sat.sat_chained(parts[r], out=parts[r], chain=chains[r], stream=streams[r])
+                    for st in streams:
+                        torch.cuda.current_stream().wait_stream(st)
+                    e1.record()
+                    torch.cuda.synchronize()
+                    if it > 0:
+                        times.append(e0.elapsed_time(e1))
+            finally:
+                sat.set_max_ctas(0)
+            slowest = max(per)
+            conc = min(times)
+            res[str(N)] = {"per_rank_ms": per, "slowest_rank_ms": slowest,
+                           "projected_efficiency": single_ms / (N * slowest),
+                           "concurrent_ms": conc, "concurrent_efficiency": single_ms / conc,
+                           "gather_path_note": "colsum + all-gather + SAT reads each element twice: <= ~0.67"}
+        finally:
+            for c in chains:
+                c.close()
+    del x
+    torch.cuda.empty_cache()
+    return res
 
 
 def run_sweep(args, sat, satgen, torch):

@@ -102,6 +102,15 @@ def build_stats(force: bool = False) -> Path:
     return out
 
 
+def build_experimental(force: bool = False) -> Path:
+    """Tuning build (-DSAT_EXPERIMENTAL=1): the shipped variants plus the unshipped configurations, for
+    tools/sweep_variants.py via SAT_LIB=paper_conf_ipps_emotofthni18_b200/libsat_exp.so.  Not the product."""
+    out = PKG / "libsat_exp.so"
+    if force or _stale(out, libsat_sources()):
+        build_libsat(extra=["-DSAT_EXPERIMENTAL=1"], out=out)
+    return out
+
+
 def build_all(force: bool = False) -> None:
     build_oracle(force)
     build_satgen(force)
@@ -110,3 +119,5 @@ def build_all(force: bool = False) -> None:
 
 if __name__ == "__main__":
     build_all(force="--force" in sys.argv)
+    if "--experimental" in sys.argv:
+        build_experimental(force="--force" in sys.argv)

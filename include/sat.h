@@ -192,6 +192,45 @@ sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, const void*
                                  void* strip_dst, int64_t strip_rows, int64_t cols, int64_t pitch,
                                  void* stream);
 
+/* ------------------------------------------------------------------ chained strip partition (NEXT-1)
+ *
+ * The same horizontal strip partition as sat_compute_sharded (rank r holds global rows
+ * [row0_r, row0_r + strip_rows)), computed in ONE pass per rank: each element is read once and written
+ * once (2 accesses instead of the 3 of colsum + all-gather + SAT).  A rank walks its strip in
+ * column-major tile order; as soon as its bottom tile of tile column J has resolved the strip's column
+ * sums over J (Step 2.B of P:198-202 restricted to the strip), its kernel pushes them -- as epoch-tagged
+ * 64-bit status words, the single-copy-atomic protocol of the look-back (R11) -- straight
+ * into the inbox of every downstream rank through peer-mapped memory over NVLink (CUDA IPC); a
+ * downstream rank's column walker adds the upstream column sums of rank 0..r-1 (ascending) to its
+ * strip-local column carry.  The column sums of tile column J arrive about one tile column of work
+ * after they are needed, well inside the pipeline's parking window, so the ranks run concurrently
+ * (DESIGN.md Sec. 7).  No NCCL call on the data path.
+ *
+ * Setup (collective, once per partition): every rank calls sat_chain_create on its own device,
+ * exports its 64-byte IPC handle with sat_chain_export, the ranks all-gather the handles (the Python
+ * binding does this over the torch process group), and every rank calls sat_chain_connect with the
+ * nranks x 64 handle bytes (its own entry is ignored).  sat_chain_connect_local instead connects n
+ * chains created in ONE process on ONE device (rank r = chains[r]): the single-GPU emulation used by
+ * the tests and by bench.py's per-rank measurements.  nranks <= 8 (one node).
+ *
+ * sat_compute_chained must be called by every rank, in the same order, with equal cols (the chain's),
+ * and >= 1 strip row per rank.  Calls are stream-ordered and asynchronous; a rank's kernel waits
+ * inside the GPU for its upstream ranks' column sums of the same call, and a rank may run at most
+ * two calls ahead of its downstream ranks (the inbox is double-buffered; back-pressure words are
+ * written by the downstream kernels at exit).  strip_src / strip_dst device (this rank), may be
+ * equal; TMA alignment rules as sat_compute.  int32 bit-exact; fp32 within the sat_compute_f32
+ * tolerance with global rows / cols.
+ * Errors: INVALID_VALUE (arguments, not connected, wrong device), OUT_OF_MEMORY, CUDA (IPC, launch),
+ * UNSUPPORTED (2^30 calls on one chain: recreate it). */
+typedef struct sat_chain_s* sat_chain_t;
+sat_status_t sat_chain_create(int nranks, int rank, int64_t cols, sat_chain_t* chain);
+sat_status_t sat_chain_export(sat_chain_t chain, unsigned char handle[64]);
+sat_status_t sat_chain_connect(sat_chain_t chain, const unsigned char* handles);
+sat_status_t sat_chain_connect_local(sat_chain_t* chains, int n);
+sat_status_t sat_chain_destroy(sat_chain_t chain);
+sat_status_t sat_compute_chained(sat_chain_t chain, sat_dtype_t dtype, const void* strip_src, void* strip_dst,
+                                 int64_t strip_rows, int64_t cols, int64_t pitch, void* stream);
+
 /* ------------------------------------------------------------------ introspection */
 
 typedef struct {

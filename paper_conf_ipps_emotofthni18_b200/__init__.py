@@ -22,6 +22,7 @@ _lib.lib()  # load now: fail loudly at import if the native library is missing
 
 __all__ = [
     "sat", "sat_batched", "sat_batched_u8", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "Chain", "sat_chained", "exchange_blobs",
     "strip_layout", "broadcast_unique_id",
     "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "debug_workspace",
     "release_stream_workspace", "release_workspaces",
@@ -323,6 +324,80 @@ def sat_sharded(strip, out=None, *, comm: Comm, stream=None, check_layout: bool 
     with torch.cuda.device(strip.device):
         check(_lib.lib().sat_compute_sharded(comm._h, _dtype_code(strip), strip.data_ptr(), out.data_ptr(), rows,
                                              cols, pitch, _stream_ptr(stream)), "sat_compute_sharded")
+    return out
+
+
+def exchange_blobs(blob: bytes, group=None) -> list[bytes]:
+    """All-gather one fixed-size byte string per rank over a torch process group (host-side plumbing of
+    the chained partition: the 64-byte CUDA IPC handles).  Works over nccl (CUDA tensors) and gloo."""
+    import torch.distributed as dist
+
+    torch = _torch()
+    world = dist.get_world_size(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if dist.get_backend(group) == "nccl" else torch.device("cpu")
+    mine = torch.tensor(list(blob), dtype=torch.uint8, device=dev)
+    allv = [torch.empty_like(mine) for _ in range(world)]
+    dist.all_gather(allv, mine, group=group)
+    return [bytes(v.cpu().tolist()) for v in allv]
+
+
+class Chain:
+    """Chained strip partition (sat_chain_*, NEXT-1): rank r's strip of a horizontally partitioned
+    matrix, computed in one pass with the strip column sums of the ranks above arriving through
+    peer-mapped memory inside the kernels.  ``Chain(cols, group=g)`` is collective over a torch process
+    group (one process per GPU; the IPC handles are all-gathered over ``g``); ``Chain.local(n, cols)``
+    builds the n ranks of an emulated chain inside ONE process on the current device."""
+
+    def __init__(self, cols: int, group=None, *, _local=None):
+        if _local is not None:
+            self.nranks, self.rank = _local
+            self.group = None
+        else:
+            import torch.distributed as dist
+
+            self.group = group
+            self.nranks, self.rank = dist.get_world_size(group), dist.get_rank(group)
+        self.cols = cols
+        self._h = ctypes.c_void_p()
+        check(_lib.lib().sat_chain_create(self.nranks, self.rank, cols, ctypes.byref(self._h)), "sat_chain_create")
+        if _local is None:
+            handle = ctypes.create_string_buffer(64)
+            check(_lib.lib().sat_chain_export(self._h, handle), "sat_chain_export")
+            blobs = exchange_blobs(handle.raw, group)
+            check(_lib.lib().sat_chain_connect(self._h, b"".join(blobs)), "sat_chain_connect")
+
+    @classmethod
+    def local(cls, n: int, cols: int) -> list["Chain"]:
+        chains = [cls(cols, _local=(n, r)) for r in range(n)]
+        arr = (ctypes.c_void_p * n)(*[c._h.value for c in chains])
+        check(_lib.lib().sat_chain_connect_local(arr, n), "sat_chain_connect_local")
+        return chains
+
+    def close(self):
+        if self._h:
+            _lib.lib().sat_chain_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def sat_chained(strip, out=None, *, chain: Chain, stream=None):
+    """This rank's strip of the SAT of the row-stacked strips of all ranks (sat_compute_chained).  Collective
+    over the chain (every rank, same order, >= 1 row each)."""
+    torch = _torch()
+    rows, cols, pitch = _matrix(strip, "strip")
+    if out is None:
+        out = torch.empty_strided((rows, cols), (pitch, 1), dtype=strip.dtype, device=strip.device)
+    orows, ocols, opitch = _matrix(out, "out")
+    if (orows, ocols, opitch) != (rows, cols, pitch) or out.dtype != strip.dtype or out.device != strip.device:
+        raise ValueError("out must match strip in shape, row stride, dtype and device")
+    with torch.cuda.device(strip.device):
+        check(_lib.lib().sat_compute_chained(chain._h, _dtype_code(strip), strip.data_ptr(), out.data_ptr(), rows, cols,
+                                             pitch, _stream_ptr(stream)), "sat_compute_chained")
     return out
 
 

@@ -25,6 +25,8 @@ EXPORTS = (
     "sat_compute_i32", "sat_compute_f32", "sat_compute_u8", "sat_compute", "sat_compute_host", "sat_compute_batched", "sat_compute_batched_u8", "sat_box_sum", "sat_rect_sums",
     "sat_strip_colsum",
     "sat_carry_prefix", "sat_comm_get_unique_id", "sat_comm_init", "sat_comm_destroy", "sat_compute_sharded",
+    "sat_chain_create", "sat_chain_export", "sat_chain_connect", "sat_chain_connect_local", "sat_chain_destroy",
+    "sat_compute_chained",
     "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order", "sat_debug_stats", "sat_debug_trace",
     "sat_debug_workspace", "sat_release_stream_workspace", "sat_release_workspaces", "sat_status_string", "sat_last_error_detail", "sat_version",
 )
@@ -70,6 +72,12 @@ def _declare(lib):
         "sat_comm_init": [ctypes.POINTER(_vp), ctypes.c_char_p, _int, _int],
         "sat_comm_destroy": [_vp],
         "sat_compute_sharded": [_vp, _int, _vp, _vp, _i64, _i64, _i64, _vp],
+        "sat_chain_create": [_int, _int, _i64, ctypes.POINTER(_vp)],
+        "sat_chain_export": [_vp, ctypes.c_char_p],
+        "sat_chain_connect": [_vp, ctypes.c_char_p],
+        "sat_chain_connect_local": [ctypes.POINTER(_vp), _int],
+        "sat_chain_destroy": [_vp],
+        "sat_compute_chained": [_vp, _int, _vp, _vp, _i64, _i64, _i64, _vp],
         "sat_query_plan": [_int, _i64, _i64, _i64, _vp, _vp, ctypes.POINTER(SatPlan)],
         "sat_set_tuning": [_int, _int, _int],
         "sat_set_max_ctas": [_int],
@@ -86,6 +94,11 @@ def _declare(lib):
         "sat_version": [],
     }
     for name, args in sig.items():
+        f = getattr(lib, name, None)
+        if f is None:
+            if not os.environ.get("SAT_LIB"):
+                raise ImportError(f"{LIB_PATH} lacks {name}: rebuild it (python build_native.py)")
+            continue  # an older tuning build named by SAT_LIB: only the calls it has
         f = getattr(lib, name)
         f.argtypes = args
         f.restype = _int

@@ -101,9 +101,10 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
 
 #endif
 
-template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC, int LB, int CT>
-struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT>> {
-    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT>;
+template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC, int LB, int CT, int DW,
+          int CH>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT, DW, CH>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT, DW, CH>;
     static constexpr int box_cols = Cfg::TB;
     static constexpr int out_box_rows = Cfg::OBR;
     static constexpr int threads = Cfg::THREADS;
@@ -133,10 +134,20 @@ struct HasU8 { static constexpr bool value = false; };
 template <typename F>
 struct HasU8<F, std::void_t<decltype(F::smem_u8())>> { static constexpr bool value = true; };
 
+template <typename Cfg, typename = void>
+struct IsChain { static constexpr bool value = false; };
+template <typename Cfg>
+struct IsChain<Cfg, std::void_t<decltype(Cfg::CHAIN)>> { static constexpr bool value = Cfg::CHAIN; };
+
 template <typename V, typename F>
 void* pick_kernel(bool tma, bool carry) {
-    return tma ? (carry ? F::template kernel<V, true, true>() : F::template kernel<V, true, false>())
-               : (carry ? F::template kernel<V, false, true>() : F::template kernel<V, false, false>());
+    if constexpr (IsChain<typename F::Cfg>::value) {  // chained strips take no carry row
+        (void)carry;
+        return tma ? F::template kernel<V, true, false>() : F::template kernel<V, false, false>();
+    } else {
+        return tma ? (carry ? F::template kernel<V, true, true>() : F::template kernel<V, true, false>())
+                   : (carry ? F::template kernel<V, false, true>() : F::template kernel<V, false, false>());
+    }
 }
 
 template <typename V, typename Cfg>
@@ -202,7 +213,7 @@ Variant make_variant() {
     v.prepare[SAT_FLOAT32] = &prepare_variant<float, Cfg>;
     if constexpr (HasBox<Family<Cfg>>::value) v.TB = Family<Cfg>::box_cols;
     else v.TB = Cfg::TC;
-    if constexpr (HasU8<Family<Cfg>>::value && Cfg::TC == 128) {
+    if constexpr (HasU8<Family<Cfg>>::value && Cfg::TC == 128 && !IsChain<Cfg>::value) {
         v.launch[kU8] = &launch_variant_u8<Cfg>;
         v.prepare[kU8] = &prepare_variant_u8<Cfg>;
     } else {
@@ -215,28 +226,36 @@ Variant make_variant() {
 // Shipped kernel variants (auto_variant picks among them; sat_set_tuning can force one, test hook).
 // Tuning builds (-DSAT_EXPERIMENTAL=1) append the configurations measured and not kept in round 1
 // (DESIGN.md Sec. 5), so that they can still be re-measured.
-enum : int { kVarClassic = 0, kVarTm128 = 1, kVarU8 = 2, kVarFlat = 3 };
+enum : int { kVarClassic = 0, kVarTm128 = 1, kVarU8 = 2, kVarFlat = 3, kVarChain = 4 };
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),                   // 0: classic, 64 x 128 tiles (small matrices)
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),                  // 1: TMEM-parked, 128 x 128 tiles
         make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>>(),                  // 2: u8 integral images (4 stages of 16 KiB)
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 3: TMEM-parked, flat 64 x 256 tiles
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 4, 0, 32, 1>>(),  // 4: chained strips (sat_compute_chained only)
 #if SAT_EXPERIMENTAL
-        make_variant<sat::TmCfg<16, 2, 5>>(),  // 4: walkers publish (blocking ws_walker)
-        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 5
-        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch>>(),  // 6: warp-specialised, TMA store
-        make_variant<sat::TmCfg<16, 2, 5, 1, 2>>(),  // 7
-        make_variant<sat::TileCfg<128, 128, 16, 2>>(),  // 8: classic, 128 x 128 tiles
-        make_variant<sat::TmCfg<16, 2, 7, 1, 1, 4>>(),  // 9
-        make_variant<sat::TmCfg<16, 3, 8, 1, 3, 4, 1>>(),  // 10: GSAT from registers
-        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 11
-        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),    // 12: flat, ring of 8
-        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 64, 256>>(),    // 13: flat, ring of 7
-        make_variant<sat::TmCfg<8, 2, 10, 1, 3, 4, 0, 0, 64, 256>>(),   // 14: flat, ring of 10
-        make_variant<sat::TmCfg<16, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),   // 15: flat, 16 compute warps
-        make_variant<sat::TmCfg<8, 3, 7, 1, 3, 4, 1, 0, 64, 256>>(),    // 16: flat, GSAT from registers
-        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 1>>(),  // 17: flat, 8 contiguous columns
+        make_variant<sat::TmCfg<16, 2, 5>>(),  // 5: walkers publish (blocking ws_walker)
+        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 6
+        make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch>>(),  // 7: warp-specialised, TMA store
+        make_variant<sat::TmCfg<16, 2, 5, 1, 2>>(),  // 8
+        make_variant<sat::TileCfg<128, 128, 16, 2>>(),  // 9: classic, 128 x 128 tiles
+        make_variant<sat::TmCfg<16, 2, 7, 1, 1, 4>>(),  // 10
+        make_variant<sat::TmCfg<16, 3, 8, 1, 3, 4, 1>>(),  // 11: GSAT from registers
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 1>>(),  // 12
+        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),    // 13: flat, ring of 8
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 64, 256>>(),    // 14: flat, ring of 7
+        make_variant<sat::TmCfg<8, 2, 10, 1, 3, 4, 0, 0, 64, 256>>(),   // 15: flat, ring of 10
+        make_variant<sat::TmCfg<16, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),   // 16: flat, 16 compute warps
+        make_variant<sat::TmCfg<8, 3, 7, 1, 3, 4, 1, 0, 64, 256>>(),    // 17: flat, GSAT from registers
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 1>>(),  // 18: flat, 8 contiguous columns
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 4>>(),         // 19: 128^2, look-back 4 per round
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8>>(),         // 20: 128^2, 8 per round
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32>>(),  // 21: ... diagonal 32 per round
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 2, 0, 32>>(),  // 22: 128^2, diagonal 32 per round
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 4>>(),           // 23: flat, look-back 4 per round
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 4, 0, 32>>(),    // 24: ... diagonal 32 per round
+        make_variant<sat::TmCfg<16, 2, 9, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32>>(),  // 25: 21 + ring of 9
 #endif
     };
     return vs;
@@ -286,14 +305,14 @@ sat_status_t device_info(int dev, DeviceInfo** out) {
 // SM count of `dev` (cached; takes g_mu)
 sat_status_t device_sms(int dev, int* sms) {
     std::lock_guard<std::mutex> lk(g_mu);
-    DeviceInfo* di;
+    DeviceInfo* di = nullptr;
     sat_status_t s = device_info(dev, &di);
     if (s == SAT_OK) *sms = di->sms;
     return s;
 }
 
 sat_status_t occupancy(int dev, int vi, int dt, bool tma, bool carry, int* occ) {
-    DeviceInfo* di;
+    DeviceInfo* di = nullptr;
     sat_status_t s = device_info(dev, &di);
     if (s != SAT_OK) return s;
     const std::pair<int, int> key(vi, dt * 4 + (tma ? 2 : 0) + (carry ? 1 : 0));
@@ -499,9 +518,12 @@ struct Plan {
 };
 
 sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* src, const void* dst, Plan* pl,
-                       bool u8 = false, int64_t src_pitch = 0) {
+                       bool u8 = false, int64_t src_pitch = 0, int force_vi = -1) {
     int vi, order;
-    {
+    if (force_vi >= 0) {
+        vi = force_vi;
+        order = 0;
+    } else {
         std::lock_guard<std::mutex> lk(g_mu);
         vi = g_variant >= 0 ? g_variant : (u8 ? kVarU8 : auto_variant(rows, cols));
         order = (g_variant < 0 && g_order == 0) ? auto_order(vi, cols) : g_order;
@@ -559,7 +581,7 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
     {
         std::lock_guard<std::mutex> lk(g_mu);
         if ((s = occupancy(dev, pl.vi, dt, pl.tma, carry != nullptr, &occ)) != SAT_OK) return s;
-        DeviceInfo* di;
+        DeviceInfo* di = nullptr;
         if ((s = device_info(dev, &di)) != SAT_OK) return s;
         sms = di->sms;
         max_ctas = g_max_ctas;
@@ -592,6 +614,7 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
         }
     }
     KParams<uint32_t> p;  // identical layout for float
+    std::memset(&p, 0, sizeof(p));  // epoch_override = 0, no chain
     p.src = static_cast<const uint32_t*>(src);
     p.dst = static_cast<uint32_t*>(dst);
     p.rows = rows;
@@ -1178,6 +1201,193 @@ SAT_API sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, con
 #endif
 }
 
+// ====================================================================== chained strip partition
+// (DESIGN.md Sec. 7): one persistent launch per rank and call, the strip column
+// sums travel rank -> downstream ranks inside the kernels through peer-mapped inbox memory.
+struct sat_chain_s {
+    std::mutex mu;
+    int nranks = 0, rank = 0, dev = 0;
+    int64_t cols = 0, inbox_cols = 0;
+    void* mem = nullptr;  // exported: inbox [2][kMaxChainRanks][inbox_cols] uint64 | done [kMaxChainRanks] uint32
+    size_t inbox_bytes = 0, mem_bytes = 0;
+    void* peer[sat::kMaxChainRanks] = {};
+    bool opened[sat::kMaxChainRanks] = {};
+    uint64_t calls = 0;
+    Ctrl* ctrl = nullptr;
+    uint64_t* slots = nullptr;
+    size_t slot_words = 0;
+};
+
+SAT_API sat_status_t sat_chain_create(int nranks, int rank, int64_t cols, sat_chain_t* out) {
+    if (!out || nranks < 1 || nranks > sat::kMaxChainRanks || rank < 0 || rank >= nranks || cols < 1 ||
+        cols > (int64_t(1) << 31) - 1)
+        return fail(SAT_ERR_INVALID_VALUE, "bad chain arguments (nranks %d, rank %d, cols %lld; nranks <= %d)", nranks,
+                    rank, (long long)cols, sat::kMaxChainRanks);
+    auto* c = new sat_chain_s();
+    c->nranks = nranks;
+    c->rank = rank;
+    c->cols = cols;
+    c->inbox_cols = (cols + 127) / 128 * 128;
+    c->inbox_bytes = static_cast<size_t>(2) * sat::kMaxChainRanks * c->inbox_cols * 8;
+    c->mem_bytes = c->inbox_bytes + 256;
+    cudaError_t e = cudaGetDevice(&c->dev);
+    if (e == cudaSuccess) e = cudaMalloc(&c->mem, c->mem_bytes);  // cudaMalloc: exportable with cudaIpcGetMemHandle
+    if (e == cudaSuccess) e = cudaMemset(c->mem, 0, c->mem_bytes);
+    if (e == cudaSuccess) e = cudaMalloc(&c->ctrl, 256);
+    if (e == cudaSuccess) e = cudaMemset(c->ctrl, 0, 256);
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        if (c->mem) cudaFree(c->mem);
+        if (c->ctrl) cudaFree(c->ctrl);
+        delete c;
+        return fail(SAT_ERR_OUT_OF_MEMORY, "chain buffers: %s", cudaGetErrorString(e));
+    }
+    c->peer[rank] = c->mem;
+    *out = c;
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_chain_export(sat_chain_t chain, unsigned char handle[64]) {
+    if (!chain || !handle) return fail(SAT_ERR_INVALID_VALUE, "null argument");
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "cudaIpcMemHandle_t size");
+    cudaIpcMemHandle_t h;
+    SAT_CUDA(cudaIpcGetMemHandle(&h, chain->mem));
+    std::memcpy(handle, &h, 64);
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_chain_connect(sat_chain_t chain, const unsigned char* handles) {
+    if (!chain || !handles) return fail(SAT_ERR_INVALID_VALUE, "null argument");
+    std::lock_guard<std::mutex> lk(chain->mu);
+    for (int g = 0; g < chain->nranks; ++g) {
+        if (g == chain->rank || chain->peer[g]) continue;
+        cudaIpcMemHandle_t h;
+        std::memcpy(&h, handles + 64 * g, 64);
+        void* ptr = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaIpcOpenMemHandle (chain peer)");
+        chain->peer[g] = ptr;
+        chain->opened[g] = true;
+    }
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_chain_connect_local(sat_chain_t* chains, int n) {
+    if (!chains || n < 1 || n > sat::kMaxChainRanks) return fail(SAT_ERR_INVALID_VALUE, "bad chain list");
+    for (int r = 0; r < n; ++r)
+        if (!chains[r] || chains[r]->nranks != n || chains[r]->rank != r || chains[r]->dev != chains[0]->dev ||
+            chains[r]->cols != chains[0]->cols)
+            return fail(SAT_ERR_INVALID_VALUE, "chains[r] must be rank r of %d on one device with equal cols", n);
+    for (int r = 0; r < n; ++r)
+        for (int g = 0; g < n; ++g) chains[r]->peer[g] = chains[g]->mem;
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_chain_destroy(sat_chain_t chain) {
+    if (!chain) return SAT_OK;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(chain->dev);
+    cudaDeviceSynchronize();
+    for (int g = 0; g < chain->nranks; ++g)
+        if (chain->opened[g]) cudaIpcCloseMemHandle(chain->peer[g]);
+    if (chain->slots) cudaFree(chain->slots);
+    if (chain->ctrl) cudaFree(chain->ctrl);
+    if (chain->mem) cudaFree(chain->mem);
+    cudaSetDevice(cur);
+    delete chain;
+    cudaGetLastError();
+    return SAT_OK;
+}
+
+SAT_API sat_status_t sat_compute_chained(sat_chain_t chain, sat_dtype_t dtype, const void* strip_src, void* strip_dst,
+                                         int64_t strip_rows, int64_t cols, int64_t pitch, void* stream) {
+    if (!chain) return fail(SAT_ERR_INVALID_VALUE, "null chain");
+    if (dtype != SAT_INT32 && dtype != SAT_FLOAT32) return fail(SAT_ERR_INVALID_VALUE, "unknown dtype %d", (int)dtype);
+    if (cols != chain->cols) return fail(SAT_ERR_INVALID_VALUE, "cols %lld != the chain's %lld", (long long)cols,
+                                         (long long)chain->cols);
+    if (strip_rows < 1) return fail(SAT_ERR_INVALID_VALUE, "chained strips need >= 1 row per rank");
+    sat_status_t s = validate(strip_src, strip_dst, strip_rows, cols, pitch);
+    if (s != SAT_OK) return s;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    std::lock_guard<std::mutex> lk(chain->mu);
+    for (int g = 0; g < chain->nranks; ++g)
+        if (!chain->peer[g]) return fail(SAT_ERR_INVALID_VALUE, "chain not connected (rank %d)", g);
+    if (chain->calls + 2 >= sat::kEpochMax) return fail(SAT_ERR_UNSUPPORTED, "chain epoch exhausted: recreate it");
+    Plan pl;
+    if ((s = make_plan(strip_rows, cols, pitch, strip_src, strip_dst, &pl, false, 0, kVarChain)) != SAT_OK) return s;
+    const Variant& v = variants()[kVarChain];
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    if (dev != chain->dev) return fail(SAT_ERR_INVALID_VALUE, "chain lives on device %d, current device %d", chain->dev, dev);
+    int occ = 0, sms = 0, max_ctas = 0;
+    {
+        std::lock_guard<std::mutex> g(g_mu);
+        if ((s = occupancy(dev, kVarChain, dtype, pl.tma, false, &occ)) != SAT_OK) return s;
+        DeviceInfo* di = nullptr;
+        if ((s = device_info(dev, &di)) != SAT_OK) return s;
+        sms = di->sms;
+        max_ctas = g_max_ctas;
+    }
+    int64_t grid = static_cast<int64_t>(sms) * occ;
+    if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
+    if (grid > pl.ntiles) grid = pl.ntiles;
+    const size_t words = static_cast<size_t>(pl.ntiles) * (v.TR + v.TC + 1);
+    if (words > chain->slot_words) {
+        const size_t want = words + words / 4;
+        if (chain->slots) SAT_CUDA(cudaFreeAsync(chain->slots, st));
+        chain->slots = nullptr;
+        chain->slot_words = 0;
+        cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&chain->slots), want * 8, st);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(SAT_ERR_OUT_OF_MEMORY, "chain slots (%zu bytes)", want * 8);
+        }
+        SAT_CUDA(cudaMemsetAsync(chain->slots, 0, want * 8, st));
+        chain->slot_words = want;
+    }
+    CUtensorMap mi, mo;
+    std::memset(&mi, 0, sizeof(mi));
+    std::memset(&mo, 0, sizeof(mo));
+    if (pl.tma) {
+        if ((s = get_encoder()) != SAT_OK) return s;
+        if ((s = encode_map(&mi, dtype, strip_src, strip_rows, cols, pitch, v.TR, v.TB)) != SAT_OK) return s;
+        if ((s = encode_map(&mo, dtype, strip_dst, strip_rows, cols, pitch, v.OBR, v.TB)) != SAT_OK) return s;
+    }
+    const uint32_t epoch = static_cast<uint32_t>(chain->calls + 1);
+    KParams<uint32_t> p;
+    std::memset(&p, 0, sizeof(p));
+    p.src = static_cast<const uint32_t*>(strip_src);
+    p.dst = static_cast<uint32_t*>(strip_dst);
+    p.rows = strip_rows;
+    p.cols = cols;
+    p.pitch = pitch;
+    p.R = pl.R;
+    p.C = pl.C;
+    p.ntiles = static_cast<int>(pl.ntiles);
+    p.order = 2;
+    p.row_slots = chain->slots;
+    p.col_slots = chain->slots + static_cast<size_t>(pl.ntiles) * v.TR;
+    p.corner_slots = chain->slots + static_cast<size_t>(pl.ntiles) * (v.TR + v.TC);
+    p.ctrl = chain->ctrl;
+    p.carry = nullptr;
+    p.src_pitch = pitch;
+    p.epoch_override = epoch;
+    p.chain.rank = chain->rank;
+    p.chain.nranks = chain->nranks;
+    p.chain.parity = epoch & 1u;
+    p.chain.inbox_cols = chain->inbox_cols;
+    for (int g = 0; g < chain->nranks; ++g) {
+        p.chain.peer_inbox[g] = static_cast<uint64_t*>(chain->peer[g]);
+        p.chain.peer_done[g] = reinterpret_cast<uint32_t*>(static_cast<char*>(chain->peer[g]) + chain->inbox_bytes);
+    }
+    cudaError_t e = v.launch[dtype](pl.tma, false, dim3(static_cast<unsigned>(grid)), st, mi, mo, &p);
+    if (e != cudaSuccess) return cuda_fail(e, "chained SAT kernel launch");
+    chain->calls++;
+    return SAT_OK;
+}
+
 SAT_API sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t cols, int64_t pitch, const void* src,
                                     const void* dst, sat_plan_t* plan) {
     if (!plan) return fail(SAT_ERR_INVALID_VALUE, "null plan");
@@ -1201,7 +1411,7 @@ SAT_API sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t col
     if (cudaGetDevice(&dev) == cudaSuccess) {
         std::lock_guard<std::mutex> lk(g_mu);
         int occ = 0;
-        DeviceInfo* di;
+        DeviceInfo* di = nullptr;
         if (occupancy(dev, pl.vi, dtype, pl.tma, false, &occ) == SAT_OK && device_info(dev, &di) == SAT_OK) {
             int per_sm = (g_ctas_per_sm > 0 && g_ctas_per_sm < occ) ? g_ctas_per_sm : occ;
             int64_t grid = static_cast<int64_t>(di->sms) * per_sm;
@@ -1219,7 +1429,8 @@ SAT_API sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm) {
 #if SAT_STATS
     if (order < 0 || (order & 15) > 1 || order > 0xffff) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
 #else
-    if (order < 0 || (order & ~0xff01) != 0) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
+    if (order < 0 || (order & ~0xff0f) != 0 || (order & 15) > 2)
+        return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
 #endif
     if (ctas_per_sm < 0) return fail(SAT_ERR_INVALID_VALUE, "ctas_per_sm < 0");
     std::lock_guard<std::mutex> lk(g_mu);
@@ -1247,7 +1458,8 @@ SAT_API sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* 
 }
 
 SAT_API sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out, void* stream) {
-    if (R <= 0 || C <= 0 || R * C > (int64_t(1) << 30) || !out || order < 0 || (order & ~0xff01) != 0)
+    if (R <= 0 || C <= 0 || R * C > (int64_t(1) << 30) || !out || order < 0 || (order & ~0xff0f) != 0 ||
+        (order & 15) > 2)
         return fail(SAT_ERR_INVALID_VALUE, "bad args");
     const int64_t n = R * C;
     int blocks = static_cast<int>((n + 255) / 256);

@@ -221,6 +221,35 @@ __device__ __forceinline__ void ld_relaxed2_p(const uint64_t* p, uint64_t& a, ui
                  : "memory");
 }
 
+// System-scope status words: the chained strip partition's inbox, written by a peer GPU over NVLink
+// (peer-mapped pointers) and polled by the owner; single-copy atomic 64-bit accesses as above.
+__device__ __forceinline__ void st_relaxed2_sys(uint64_t* p, uint64_t a, uint64_t b) {
+    asm volatile("st.relaxed.sys.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ void ld_relaxed2_sys(const uint64_t* p, uint64_t& a, uint64_t& b) {
+    asm volatile("ld.relaxed.sys.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void st_relaxed_sys_u32(uint32_t* p, uint32_t a) {
+    asm volatile("st.relaxed.sys.global.b32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_relaxed_sys_u32(const uint32_t* p) {
+    uint32_t a;
+    asm volatile("ld.relaxed.sys.global.b32 %0, [%1];" : "=r"(a) : "l"(p) : "memory");
+    return a;
+}
+template <int E>
+__device__ __forceinline__ void st_words_sys(uint64_t* p, const uint64_t (&w)[E]) {
+    static_assert(E % 2 == 0, "16-byte aligned word pairs");
+#pragma unroll
+    for (int e = 0; e < E; e += 2) st_relaxed2_sys(p + e, w[e], w[e + 1]);
+}
+template <int E>
+__device__ __forceinline__ void ld_words_sys(const uint64_t* p, uint64_t (&w)[E]) {
+    static_assert(E % 2 == 0, "16-byte aligned word pairs");
+#pragma unroll
+    for (int e = 0; e < E; e += 2) ld_relaxed2_sys(p + e, w[e], w[e + 1]);
+}
+
 template <int E>
 __device__ __forceinline__ void st_words_p(uint64_t* p, const uint64_t (&w)[E], uint64_t pol) {
     if constexpr (E % 2 != 0) {  // odd vectors are not 16-byte aligned per lane: scalar accesses

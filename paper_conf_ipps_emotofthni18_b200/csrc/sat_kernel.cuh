@@ -63,6 +63,19 @@ struct Ctrl {
     unsigned int pad;
 };
 
+// Chained strip partition (sat_compute_chained): rank r's
+// strip takes its column carry from the strip column sums of every rank g < r, which rank g pushes
+// (as epoch-tagged status words, prefix form over each tile's columns) into rank r's inbox over
+// NVLink peer memory as soon as its bottom tile of that tile column resolves.
+constexpr int kMaxChainRanks = 8;
+struct ChainParams {
+    int rank, nranks;
+    uint32_t parity;                         // inbox half of this call (epoch & 1)
+    int64_t inbox_cols;                      // words per inbox vector (>= C * TC)
+    uint64_t* peer_inbox[kMaxChainRanks];    // inbox of every rank: [2][kMaxChainRanks][inbox_cols] words
+    uint32_t* peer_done[kMaxChainRanks];     // back-pressure words of every rank: [kMaxChainRanks]
+};
+
 template <typename V>
 struct KParams {
     const V* src;  // generic path only
@@ -80,6 +93,8 @@ struct KParams {
     long long* trace;  // [ntiles][2]: acquisition / store-issue globaltimer ns (SAT_STATS builds only)
     const uint8_t* src8;  // u8 input (integral images, sat_compute_u8): generic path only, else nullptr
     int64_t src_pitch;    // row stride of src8 in bytes
+    uint32_t epoch_override;  // != 0: the launch epoch chosen by the host (chained calls); ctrl->epoch untouched
+    ChainParams chain;        // chained strip partition only
 };
 
 __device__ __forceinline__ uint64_t pack(uint32_t epoch, uint32_t kind, uint32_t bits) {
@@ -126,7 +141,7 @@ __device__ __forceinline__ void diag_of_serial(long long s, int R, int C, int& I
     J = static_cast<int>(d - I);
 }
 
-// order & 15: 0 = anti-diagonal (Fig. 9), 1 = row-major.  (order >> 8) & 255 = g > 1 with order & 15
+// order & 15: 0 = anti-diagonal (Fig. 9), 1 = row-major, 2 = column-major.  (order >> 8) & 255 = g > 1 with order & 15
 // == 0 and g | C: anti-diagonal order of g-wide tile groups, the g tiles of a group consecutive and
 // left to right (a topological order too: a tile's left neighbour is earlier in its group or on the
 // previous group diagonal, its upper neighbours on the previous group diagonal).  The g tiles of a
@@ -135,6 +150,11 @@ __device__ __forceinline__ void tile_of_serial(int s_, int R, int C, int order, 
     if ((order & 15) == 1) {
         I = s_ / C;
         J = s_ - I * C;
+        return;
+    }
+    if ((order & 15) == 2) {  // column-major (chained strips: a tile column's tiles are consecutive)
+        J = s_ / R;
+        I = s_ - J * R;
         return;
     }
     const int g = (order >> 8) & 255;

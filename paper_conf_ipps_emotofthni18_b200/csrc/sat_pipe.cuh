@@ -97,8 +97,11 @@ __device__ __forceinline__ void ws_exit(const KParams<V>& p, uint32_t epoch) {
     if (done == gridDim.x - 1) {
         p.ctrl->counter = 0u;
         p.ctrl->exit_count = 0u;
-        p.ctrl->epoch = (epoch >= kEpochMax) ? 1u : epoch + 1u;
+        if (p.epoch_override == 0u) p.ctrl->epoch = (epoch >= kEpochMax) ? 1u : epoch + 1u;
         __threadfence();
+        // chained strips: every CTA of this rank is done reading its inbox for this call; tell the
+        // upstream ranks, which may then reuse this parity of the inbox two calls later
+        for (int g = 0; g < p.chain.rank; ++g) st_relaxed_sys_u32(p.chain.peer_done[g] + p.chain.rank, epoch);
     }
 }
 

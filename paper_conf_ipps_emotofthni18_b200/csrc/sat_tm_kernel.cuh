@@ -32,8 +32,13 @@ namespace sat {
 // TR_ x TC_ tiles: TC_ = 128 * G (a lane owns G chunks of 4 columns, 128 apart); flat tiles (TC_ > 128)
 // keep the tile's 64 KiB but make every DRAM row visit 4 B * TC_ long (tile shape).
 template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0, int QS_ = 0,
-          int TR_ = 128, int TC_ = 128, int LB_ = 2, int CT_ = 0>
+          int TR_ = 128, int TC_ = 128, int LB_ = 2, int CT_ = 0, int DW_ = 4, int CH_ = 0>
 struct TmCfg {
+    // Chained strip partition (sat_compute_chained): column-major tile order, column carries = strip-local
+    // vertical look-back + the upstream ranks' strip column sums from the inbox, corners by a horizontal
+    // look-back; bottom tiles push their strip column sums to the downstream ranks.
+    static constexpr bool CHAIN = CH_ != 0;
+    static constexpr int DW = DW_;                  // diagonal look-back: corner words polled per round (<= 32)
     static constexpr bool CT = CT_ != 0;            // a lane owns 4 G contiguous columns (one warp scan per row)
     static constexpr int LB = LB_;                  // row / column look-back: predecessors polled per round
     static constexpr int TR = TR_, TC = TC_, NW = NW_;
@@ -66,6 +71,7 @@ struct TmCfg {
     static_assert(!SBAND || !QS, "flat tiles: whole-tile TMA stores");
     static_assert(!CT || (TC == 256 && !DIRECT), "contiguous lane columns: 64 x 256 tiles");
     static_assert(D >= 2 && D * TM_COLS_PER_SLOT <= 512, "TMEM columns");
+    static_assert(DW >= 1 && DW <= 32 && (DW & (DW - 1)) == 0, "diagonal window: a power of two <= 32");
     static_assert(IN >= 1 && NQ >= IN + D - 1 && NQ <= 16, "rings");
 #if !SAT_EXPERIMENTAL
     static_assert(DECOUPLED, "product builds ship the decoupled walkers only (-DSAT_EXPERIMENTAL=1 for the rest)");
@@ -456,7 +462,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
                     st_relaxed2_p(rs + r, pack(epoch, kIncl, to_bits(v[r][X - 1] + sm.rp[tq.s][row0 + r])),
                                   pack(epoch, kIncl, to_bits(v[r + 1][X - 1] + sm.rp[tq.s][row0 + r + 1])), pol);
             }
-            if (warp == NW - 1) {
+            if (!Cfg::CHAIN && warp == NW - 1) {  // chained strips: the column walker publishes these
                 const int cd = __shfl_sync(kFull, *reinterpret_cast<volatile int*>(&sm.cdone[tq.s]), 0);
                 if (cd == tq.k + 1) {
                     __threadfence_block();
@@ -672,6 +678,60 @@ __device__ __forceinline__ bool lb_consume_n(uint32_t& pending, int& pos, V (&ac
     return progress;
 }
 
+// Chained strips (Cfg::CHAIN), column walker, once the strip-local column look-back of tile (I,J) has
+// resolved (acc = prefix_j of the column sums of this strip's rows above the tile, VP):
+//  1. the strip-local inclusive column words VP + LCS(I,J) (Step 2.B.3 within the strip), once the owning
+//     compute warp has written its local column aggregates;
+//  2. bottom tile row: those words are this strip's column sums over tile column J -- pushed into the
+//     inbox of every downstream rank (system-scope stores to peer memory), after the downstream ranks
+//     have released this inbox half (back-pressure: they finished call epoch - 2);
+//  3. acc += the strip column sums of every upstream rank g < rank from this rank's inbox (ascending g,
+//     so fp32 sums are associated the same way on every rank): acc = prefix_j GCS(I-1,J) of the full
+//     matrix, the column carry of Step 4 (the virtual tile row above the strip, R12).
+template <typename V, typename Cfg, typename SM>
+__device__ __forceinline__ void tm_chain_column(SM& sm, const KParams<V>& p, int s, int k, int I, int J,
+                                                V (&acc)[Cfg::EC], uint64_t* own, uint32_t epoch, int lane, bool& bp_ok) {
+    constexpr int E = Cfg::EC, NW = Cfg::NW, TC = Cfg::TC;
+    const uint64_t pol = policy_evict_last();
+    const ChainParams& ch = p.chain;
+    while (*reinterpret_cast<const volatile int*>(&sm.lw[s][NW - 1]) != k + 1) __nanosleep(20);
+    __threadfence_block();
+    uint64_t wv[E];
+#pragma unroll
+    for (int e = 0; e < E; ++e) wv[e] = pack(epoch, kIncl, to_bits(sm.lcs[s][lane * E + e] + acc[e]));
+    if (I > 0) st_words_p<E>(own + lane * E, wv, pol);  // I == 0: published inclusive by the compute warp
+    const long long col = static_cast<long long>(J) * TC + lane * E;
+    if (I == p.R - 1 && ch.rank + 1 < ch.nranks) {
+        if (!bp_ok) {
+            for (int r = ch.rank + 1 + lane; r < ch.nranks; r += 32)
+                while (static_cast<long long>(ld_relaxed_sys_u32(ch.peer_done[ch.rank] + r)) <
+                       static_cast<long long>(epoch) - 2)
+                    __nanosleep(64);
+            __syncwarp();
+            bp_ok = true;
+        }
+        for (int r = ch.rank + 1; r < ch.nranks; ++r)
+            st_words_sys<E>(ch.peer_inbox[r] + (static_cast<long long>(ch.parity) * kMaxChainRanks + ch.rank) *
+                                                   ch.inbox_cols + col, wv);
+    }
+    if (ch.rank > 0) {
+        const uint64_t* inbox = ch.peer_inbox[ch.rank] + static_cast<long long>(ch.parity) * kMaxChainRanks * ch.inbox_cols + col;
+        for (int g = 0; g < ch.rank; ++g) {
+            uint64_t w[E];
+            while (true) {
+                ld_words_sys<E>(inbox + static_cast<long long>(g) * ch.inbox_cols, w);
+                bool ok = true;
+#pragma unroll
+                for (int e = 0; e < E; ++e) ok = ok && word_ready(w[e], epoch);
+                if (__all_sync(kFull, ok)) break;
+                __nanosleep(64);
+            }
+#pragma unroll
+            for (int e = 0; e < E; ++e) acc[e] = acc[e] + from_bits<V>(static_cast<uint32_t>(w[e]));
+        }
+    }
+}
+
 // Walker with a decoupled diagonal look-back (Cfg::DECOUPLED), one tile at a time, in acquisition order.
 //
 // Row walker: row look-back (Step 2.A.2) and diagonal look-back (Step 3.2).  Column
@@ -695,11 +755,12 @@ template <typename V, typename Cfg, bool ROW, typename TIn>
 __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, RPW = Cfg::RPW, NW = Cfg::NW;
     constexpr int E = ROW ? Cfg::ER : Cfg::EC;
-    constexpr int DW = 4;  // diagonal predecessors polled per round
+    constexpr int DW = Cfg::DW;  // diagonal predecessors polled per round
     // predecessors polled per round: LB, capped at 32 words (64 registers) per lane
     constexpr int NP = Cfg::LB * E <= 32 ? Cfg::LB : (32 / E >= 1 ? 32 / E : 1);
     const uint64_t pol = policy_evict_last();
     auto flag = [&](const int* f) { return *reinterpret_cast<const volatile int*>(f); };
+    bool bp_ok = false;  // chain mode: the downstream ranks have released this call's inbox half
     for (Slot<Cfg::NQ> nx;; nx.next()) {
         if (!wait_acquired(sm, nx.s, nx.ph, nx.k)) break;
         const TileInfo ti = sm.info[nx.s];
@@ -713,7 +774,8 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
         V acc[E];
 #pragma unroll
         for (int e = 0; e < E; ++e) acc[e] = V(0);
-        bool ddone = ROW ? (I == 0 || J == 0) : true;
+        // diagonal look-back (Step 3.2) -- in chain mode a horizontal one over the corner words X / XG
+        bool ddone = ROW ? (Cfg::CHAIN ? J == 0 : (I == 0 || J == 0)) : true;
 #if SAT_STATS
         if (p.order & 16) { pend = 0u; ddone = true; }  // timing experiment only: no look-back (wrong sums)
 #endif
@@ -731,8 +793,9 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                     if (pos - h >= 0) ld_words_p<E>(q - h * step, w[h], pol);
             }
             const int kk = dbase + lane;
-            const bool dinr = ROW && !ddone && lane < DW && (I - kk >= 0) && (J - kk >= 0);
-            if (dinr) wd = ld_relaxed_p(p.corner_slots + static_cast<long long>(I - kk) * p.C + (J - kk), pol);
+            const int dI = Cfg::CHAIN ? I : I - kk;
+            const bool dinr = ROW && !ddone && lane < DW && (dI >= 0) && (J - kk >= 0);
+            if (dinr) wd = ld_relaxed_p(p.corner_slots + static_cast<long long>(dI) * p.C + (J - kk), pol);
             // ---- consume
             bool progress = false;
             if (pend) progress = lb_consume_n<V, E, NP>(pend, pos, acc, w, epoch);
@@ -751,6 +814,10 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                     progress = true;
                 }
             }
+            if constexpr (Cfg::CHAIN && !ROW) {
+                if (!cin && __all_sync(kFull, pend == 0u)) tm_chain_column<V, Cfg>(sm, p, s, k, I, J, acc, own, epoch, lane,
+                                                                                    bp_ok);
+            }
             if (!cin && __all_sync(kFull, pend == 0u)) {
                 // carries -> smem, raise the flag, then publish the inclusive words of the rows / columns
                 // whose local aggregates are already in
@@ -759,12 +826,14 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                     if (ROW) sm.rp[s][lane * E + e] = acc[e];
                     else sm.cp[s][lane * E + e] = acc[e];
                 }
+                if (Cfg::CHAIN && !ROW && lane == 31)  // X(I,J): local corner word (inclusive on the left edge)
+                    st_relaxed_p(p.corner_slots + tidx, pack(epoch, J == 0 ? kIncl : kLocal, to_bits(acc[E - 1])), pol);
                 __syncwarp();
                 __threadfence_block();
                 if (lane == 0) *reinterpret_cast<volatile int*>(ROW ? &sm.rres[s] : &sm.cdone[s]) = k + 1;
                 __threadfence_block();
                 const int owner = ROW ? (lane * E) / RPW : NW - 1;  // compute warp holding these locals
-                if ((ROW ? J > 0 : I > 0) && flag(&sm.lw[s][owner]) == k + 1) {
+                if ((ROW ? J > 0 : (I > 0 && !Cfg::CHAIN)) && flag(&sm.lw[s][owner]) == k + 1) {
                     __threadfence_block();
                     uint64_t wv[E];
 #pragma unroll
@@ -777,7 +846,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                 cin = true;
                 progress = true;
             }
-            if (ROW && cin && !ddone && !lpub) {  // Step 3.1: GLS, published as a local corner word
+            if (!Cfg::CHAIN && ROW && cin && !ddone && !lpub) {  // Step 3.1: GLS, published as a local corner word
                 int go = 0;
                 if (lane == 31 && flag(&sm.cdone[s]) == k + 1 && flag(&sm.lw[s][NW - 1]) == k + 1) {
                     __threadfence_block();
@@ -791,7 +860,19 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
             if (!progress) __nanosleep(32);
         }
         // ---- Step 3.3 (GS, by whoever comes last) and the hand-off
-        if (ROW) {
+        if (ROW && Cfg::CHAIN) {
+            // corner = GS(I-1,J-1) = sum of X(I,J') over J' < J; then XG(I,J) = corner + X(I,J) = GS(I-1,J),
+            // once the column walker has published X (it never waits for this warp)
+            if (lane == 0) sm.corner[s] = dacc;
+            __syncwarp();
+            __threadfence_block();
+            if (lane == 0) *reinterpret_cast<volatile int*>(&sm.rdone[s]) = k + 1;
+            if (J > 0) {
+                while (flag(&sm.cdone[s]) != k + 1) __nanosleep(20);
+                __threadfence_block();
+                if (lane == 31) st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(dacc + sm.cp[s][TC - 1])), pol);
+            }
+        } else if (ROW) {
             if (lane == 0) sm.corner[s] = dacc;
             __syncwarp();
             __threadfence_block();
@@ -802,7 +883,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                 const V gs = dacc + ((sm.lrs[s][TR - 1] + acc[E - 1]) + sm.cp[s][TC - 1]);
                 st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(gs)), pol);
             }
-        } else {
+        } else if (!Cfg::CHAIN) {
             if (lane == 31 && flag(&sm.rdone[s]) == k + 1 && flag(&sm.lw[s][NW - 1]) == k + 1) {
                 __threadfence_block();
                 const V gs = sm.corner[s] + ((sm.lrs[s][TR - 1] + sm.rp[s][TR - 1]) + acc[E - 1]);
@@ -832,7 +913,7 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
 #endif
     if (warp == 0) tmem_alloc(&sm.tmem_base, Cfg::TM_COLS);
     if (threadIdx.x == 32) {
-        sm.epoch = *reinterpret_cast<volatile unsigned int*>(&p.ctrl->epoch);
+        sm.epoch = p.epoch_override ? p.epoch_override : *reinterpret_cast<volatile unsigned int*>(&p.ctrl->epoch);
         sm.end_n = 0x7fffffff;
 #pragma unroll
         for (int q = 0; q < Cfg::NQ; ++q) {
@@ -973,7 +1054,7 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 const int t = static_cast<int>(atomicAdd(&p.ctrl->counter, 1u));
                 const bool valid = t < p.ntiles;
                 TileInfo ti{t, 0, 0, 0};
-                if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
+                if (valid) tile_of_serial(t, p.R, p.C, Cfg::CHAIN ? 2 : p.order, ti.I, ti.J);
                 sm.info[ta.s] = ti;
                 if (!valid) {
                     *reinterpret_cast<volatile int*>(&sm.end_n) = ta.k;

@@ -61,7 +61,7 @@ def test_variants_and_tuning(sat):
     with pytest.raises(sat.SatError):
         sat.set_tuning(n, 0, 0)
     with pytest.raises(sat.SatError):
-        sat.set_tuning(-1, 2, 0)
+        sat.set_tuning(-1, 3, 0)
     with pytest.raises(sat.SatError):
         sat.set_tuning(-1, 0x201 | 0x10000, 0)
     sat.set_tuning(-1, 0x200, 0)  # anti-diagonal order of 2-tile groups

@@ -116,3 +116,48 @@ def test_strip_layout_consistent_and_mismatch():
 @pytest.mark.parametrize("world", [2, 3])
 def test_carry_exchange_protocol_gloo(world):
     _run(world, _w_carry_exchange, 61, 45, 1447 + world)
+
+
+# ----------------------------------------------------------------------------- chained partition: handle exchange
+def _blob_worker(rank, port, q):
+    try:
+        import os
+        import sys
+        from pathlib import Path
+
+        sys.path.insert(0, str(Path(__file__).resolve().parent.parent))
+        import torch.distributed as dist
+
+        import paper_conf_ipps_emotofthni18_b200 as sat
+
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+        dist.init_process_group("gloo", rank=rank, world_size=2)
+        blob = bytes((rank * 37 + i) % 256 for i in range(64))  # stands in for a 64-byte CUDA IPC handle
+        got = sat.exchange_blobs(blob, None)
+        dist.destroy_process_group()
+        q.put((rank, got))
+    except Exception:
+        import traceback
+
+        q.put((rank, traceback.format_exc()))
+
+
+def test_chain_handle_exchange_gloo_world2():
+    """The host plumbing of Chain(group): every rank receives every rank's 64-byte handle, in rank order."""
+    import socket
+
+    import torch.multiprocessing as mp
+
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_blob_worker, args=(r, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=120) for _ in range(2))
+    for p in procs:
+        p.join(timeout=30)
+    want = [bytes((r * 37 + i) % 256 for i in range(64)) for r in range(2)]
+    assert out[0] == want and out[1] == want
