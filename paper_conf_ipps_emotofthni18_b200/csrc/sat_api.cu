@@ -4,6 +4,7 @@
 #include <dlfcn.h>
 
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <map>
@@ -196,7 +197,7 @@ cudaError_t prepare_variant_u8(bool tma, bool carry, int* occupancy) {
     return cudaOccupancyMaxActiveBlocksPerMultiprocessor(occupancy, k, F::threads, smem);
 }
 
-template <typename Cfg>
+template <typename Cfg, bool U8 = false>
 Variant make_variant() {
     Variant v;
     v.TR = Cfg::TR;
@@ -213,7 +214,7 @@ Variant make_variant() {
     v.prepare[SAT_FLOAT32] = &prepare_variant<float, Cfg>;
     if constexpr (HasBox<Family<Cfg>>::value) v.TB = Family<Cfg>::box_cols;
     else v.TB = Cfg::TC;
-    if constexpr (HasU8<Family<Cfg>>::value && Cfg::TC == 128 && !IsChain<Cfg>::value) {
+    if constexpr (U8 && HasU8<Family<Cfg>>::value && Cfg::TC == 128 && !IsChain<Cfg>::value) {
         v.launch[kU8] = &launch_variant_u8<Cfg>;
         v.prepare[kU8] = &prepare_variant_u8<Cfg>;
     } else {
@@ -230,10 +231,16 @@ enum : int { kVarClassic = 0, kVarTm128 = 1, kVarU8 = 2, kVarFlat = 3, kVarChain
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),                   // 0: classic, 64 x 128 tiles (small matrices)
-        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>>(),                  // 1: TMEM-parked, 128 x 128 tiles
-        make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>>(),                  // 2: u8 integral images (4 stages of 16 KiB)
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>, true>(),            // 1: TMEM-parked, 128 x 128 tiles
+        make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>, true>(),            // 2: u8 integral images (4 stages of 16 KiB)
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 3: TMEM-parked, flat 64 x 256 tiles
-        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 4, 0, 32, 1>>(),  // 4: chained strips (sat_compute_chained only)
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32, 1>>(),  // 4: chained strips (sat_compute_chained only)
+        // round-2 candidates (medium sizes): 8 compute warps on 128 x 128 tiles, wider look-back windows
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 2>>(),            // 5
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 4, 0, 32>>(),     // 6
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32>>(),     // 7
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 4>>(),      // 8
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 0, 32>>(),      // 9: flat, diagonal 32
 #if SAT_EXPERIMENTAL
         make_variant<sat::TmCfg<16, 2, 5>>(),  // 5: walkers publish (blocking ws_walker)
         make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 6

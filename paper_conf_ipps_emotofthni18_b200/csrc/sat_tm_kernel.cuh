@@ -716,18 +716,38 @@ __device__ __forceinline__ void tm_chain_column(SM& sm, const KParams<V>& p, int
     }
     if (ch.rank > 0) {
         const uint64_t* inbox = ch.peer_inbox[ch.rank] + static_cast<long long>(ch.parity) * kMaxChainRanks * ch.inbox_cols + col;
-        for (int g = 0; g < ch.rank; ++g) {
-            uint64_t w[E];
+        // upstream ranks in groups of 4: each poll round loads every vector of the group still missing;
+        // a group is added (in ascending g) once all of it is in
+        for (int g0 = 0; g0 < ch.rank; g0 += 4) {
+            const int ng = ch.rank - g0 < 4 ? ch.rank - g0 : 4;
+            uint32_t pend = (1u << ng) - 1u;
+            V part[4][E];
             while (true) {
-                ld_words_sys<E>(inbox + static_cast<long long>(g) * ch.inbox_cols, w);
-                bool ok = true;
+                uint64_t w[4][E];
 #pragma unroll
-                for (int e = 0; e < E; ++e) ok = ok && word_ready(w[e], epoch);
-                if (__all_sync(kFull, ok)) break;
+                for (int h = 0; h < 4; ++h)
+                    if ((pend >> h) & 1u) ld_words_sys<E>(inbox + static_cast<long long>(g0 + h) * ch.inbox_cols, w[h]);
+#pragma unroll
+                for (int h = 0; h < 4; ++h) {
+                    if ((pend >> h) & 1u) {
+                        bool ok = true;
+#pragma unroll
+                        for (int e = 0; e < E; ++e) ok = ok && word_ready(w[h][e], epoch);
+                        if (__all_sync(kFull, ok)) {
+#pragma unroll
+                            for (int e = 0; e < E; ++e) part[h][e] = from_bits<V>(static_cast<uint32_t>(w[h][e]));
+                            pend &= ~(1u << h);
+                        }
+                    }
+                }
+                if (!pend) break;
                 __nanosleep(64);
             }
 #pragma unroll
-            for (int e = 0; e < E; ++e) acc[e] = acc[e] + from_bits<V>(static_cast<uint32_t>(w[e]));
+            for (int h = 0; h < 4; ++h)
+                if (h < ng)
+#pragma unroll
+                    for (int e = 0; e < E; ++e) acc[e] = acc[e] + part[h][e];
         }
     }
 }
