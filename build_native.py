@@ -111,10 +111,26 @@ def build_experimental(force: bool = False) -> Path:
     return out
 
 
+def build_stress(force: bool = False) -> Path:
+    """Protocol-stress build: -DSAT_JITTER=1 (random __nanosleep before every status-word
+    publication) and -DSAT_WATCHDOG=1 (bounded spins that trap).  For tests/test_gpu_stress.py via
+    SAT_LIB=paper_conf_ipps_emotofthni18_b200/libsat_stress.so.  Not the product."""
+    out = PKG / "libsat_stress.so"
+    if force or _stale(out, libsat_sources()):
+        build_libsat(extra=["-DSAT_JITTER=1", "-DSAT_WATCHDOG=1"], out=out)
+    return out
+
+
 def build_all(force: bool = False) -> None:
+    """Oracle, generators, libsat.so and the protocol-stress build (the two nvcc runs in parallel)."""
+    from concurrent.futures import ThreadPoolExecutor
+
     build_oracle(force)
     build_satgen(force)
-    build_libsat(force)
+    with ThreadPoolExecutor(2) as ex:
+        jobs = [ex.submit(build_libsat, force), ex.submit(build_stress, force)]
+        for j in jobs:
+            j.result()
 
 
 if __name__ == "__main__":

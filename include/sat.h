@@ -268,6 +268,14 @@ sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* tile_col
  * out: device int32[2*R*C], out[2s] = I, out[2s+1] = J of serial s. */
 sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out, void* stream);
 
+/* Test hook: launch `ctas` CTAs on `stream` that each hold `smem_bytes` (<= 227 KiB) of shared memory and
+ * spin for `ns` (<= 1e10) nanoseconds.  With ctas close to the SM count and smem_bytes large enough that a
+ * SAT CTA cannot share an SM, a SAT launched next on another stream starts with only a few resident
+ * CTAs and gets the rest as the occupying CTAs retire: the forward-progress condition of P:21 / the
+ * SKSS counter under an adversarial CTA -> SM assignment.  INVALID_VALUE on bad arguments,
+ * SAT_ERR_CUDA on a launch error. */
+sat_status_t sat_debug_occupy(int ctas, int64_t ns, int64_t smem_bytes, void* stream);
+
 /* Test/tuning hook: per-CTA phase counters (cycles, look-back steps) of the most recent launch.
  * out: host int64[max_ctas * n_stats].  Only libsat_stats.so (built with -DSAT_STATS=1) records
  * them; the production library returns SAT_ERR_UNSUPPORTED. */

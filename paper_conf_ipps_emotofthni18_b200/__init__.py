@@ -24,7 +24,7 @@ __all__ = [
     "sat", "sat_batched", "sat_batched_u8", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
     "Chain", "sat_chained", "exchange_blobs",
     "strip_layout", "broadcast_unique_id",
-    "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "debug_workspace",
+    "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "debug_occupy", "debug_workspace",
     "release_stream_workspace", "release_workspaces",
     "version", "SatError", "SAT_INT32", "SAT_FLOAT32",
 ]
@@ -436,6 +436,12 @@ def debug_tile_order(R: int, C: int, order: int = 0, device=None):
     with torch.cuda.device(out.device):
         check(_lib.lib().sat_debug_tile_order(R, C, order, out.data_ptr(), _stream_ptr(None)), "sat_debug_tile_order")
     return out
+
+
+def debug_occupy(ctas: int, ns: int, smem_bytes: int = 200 * 1024, *, stream=None) -> None:
+    """Test hook (sat_debug_occupy): ``ctas`` CTAs holding ``smem_bytes`` of shared memory each spin for
+    ``ns`` nanoseconds on ``stream`` (adversarial SM occupancy for the forward-progress tests)."""
+    check(_lib.lib().sat_debug_occupy(ctas, ns, smem_bytes, _stream_ptr(stream)), "sat_debug_occupy")
 
 
 def debug_workspace(stream=None, words: bool = True):

@@ -27,7 +27,7 @@ EXPORTS = (
     "sat_carry_prefix", "sat_comm_get_unique_id", "sat_comm_init", "sat_comm_destroy", "sat_compute_sharded",
     "sat_chain_create", "sat_chain_export", "sat_chain_connect", "sat_chain_connect_local", "sat_chain_destroy",
     "sat_compute_chained",
-    "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order", "sat_debug_stats", "sat_debug_trace",
+    "sat_query_plan", "sat_set_tuning", "sat_set_max_ctas", "sat_num_variants", "sat_variant_info", "sat_debug_tile_order", "sat_debug_occupy", "sat_debug_stats", "sat_debug_trace",
     "sat_debug_workspace", "sat_release_stream_workspace", "sat_release_workspaces", "sat_status_string", "sat_last_error_detail", "sat_version",
 )
 
@@ -84,6 +84,7 @@ def _declare(lib):
         "sat_num_variants": [],
         "sat_variant_info": [_int, ctypes.POINTER(_i32), ctypes.POINTER(_i32)],
         "sat_debug_tile_order": [_i64, _i64, _int, _vp, _vp],
+        "sat_debug_occupy": [_int, _i64, _i64, _vp],
         "sat_debug_stats": [_vp, _int, ctypes.POINTER(_int), ctypes.POINTER(_int)],
         "sat_debug_trace": [_vp, _i64, ctypes.POINTER(_i64)],
         "sat_debug_workspace": [_vp, _vp, _i64, ctypes.POINTER(SatWsInfo)],

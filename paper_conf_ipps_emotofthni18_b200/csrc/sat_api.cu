@@ -67,6 +67,7 @@ struct Variant {
     int TB;                // TMA box width in elements (TC, or 256 for flat tiles: NB = TC / TB boxes)
     int OBR;               // rows of the output TMA box (TR, or TR/4 for quarter stores)
     int family;            // 2 = TMEM-parked (sat_tm_kernel), 1 = warp-specialised (sat_ws_kernel), 0 = classic
+    bool chain;            // chained-strip configuration (sat_compute_chained only)
     size_t smem;           // dynamic shared memory bytes (same for int32 / fp32)
     LaunchFn launch[3];    // [dtype]; [kU8] = u8 input -> uint32 SAT (TMEM-parked family only, else null)
     PrepareFn prepare[3];  // [dtype]
@@ -205,6 +206,7 @@ Variant make_variant() {
     v.NW = Cfg::NW;
     v.STAGES = Cfg::STAGES;
     v.family = Family<Cfg>::family;
+    v.chain = IsChain<Cfg>::value;
     if constexpr (HasOBR<Family<Cfg>>::value) v.OBR = Family<Cfg>::out_box_rows;
     else v.OBR = Cfg::TR;
     v.smem = Family<Cfg>::template smem<uint32_t>();
@@ -263,6 +265,7 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 4>>(),           // 23: flat, look-back 4 per round
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 4, 0, 32>>(),    // 24: ... diagonal 32 per round
         make_variant<sat::TmCfg<16, 2, 9, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32>>(),  // 25: 21 + ring of 9
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 4, 0, 32, 1>>(),   // 26: chained strips, flat 64 x 256
 #endif
     };
     return vs;
@@ -532,8 +535,9 @@ sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* sr
         order = 0;
     } else {
         std::lock_guard<std::mutex> lk(g_mu);
-        vi = g_variant >= 0 ? g_variant : (u8 ? kVarU8 : auto_variant(rows, cols));
-        order = (g_variant < 0 && g_order == 0) ? auto_order(vi, cols) : g_order;
+        const bool forced = g_variant >= 0 && !variants()[g_variant].chain;  // chain configs: chained calls only
+        vi = forced ? g_variant : (u8 ? kVarU8 : auto_variant(rows, cols));
+        order = (!forced && g_order == 0) ? auto_order(vi, cols) : g_order;
     }
     const Variant& v = variants()[vi];
     pl->vi = vi;
@@ -1215,7 +1219,7 @@ struct sat_chain_s {
     std::mutex mu;
     int nranks = 0, rank = 0, dev = 0;
     int64_t cols = 0, inbox_cols = 0;
-    void* mem = nullptr;  // exported: inbox [2][kMaxChainRanks][inbox_cols] uint64 | done [kMaxChainRanks] uint32
+    void* mem = nullptr;  // exported: inbox [2][inbox_cols] uint64 | done [kMaxChainRanks] uint32
     size_t inbox_bytes = 0, mem_bytes = 0;
     void* peer[sat::kMaxChainRanks] = {};
     bool opened[sat::kMaxChainRanks] = {};
@@ -1234,8 +1238,8 @@ SAT_API sat_status_t sat_chain_create(int nranks, int rank, int64_t cols, sat_ch
     c->nranks = nranks;
     c->rank = rank;
     c->cols = cols;
-    c->inbox_cols = (cols + 127) / 128 * 128;
-    c->inbox_bytes = static_cast<size_t>(2) * sat::kMaxChainRanks * c->inbox_cols * 8;
+    c->inbox_cols = (cols + 255) / 256 * 256;  // whole tiles of the widest chain configuration (TC = 256)
+    c->inbox_bytes = static_cast<size_t>(2) * c->inbox_cols * 8;
     c->mem_bytes = c->inbox_bytes + 256;
     cudaError_t e = cudaGetDevice(&c->dev);
     if (e == cudaSuccess) e = cudaMalloc(&c->mem, c->mem_bytes);  // cudaMalloc: exportable with cudaIpcGetMemHandle
@@ -1308,6 +1312,18 @@ SAT_API sat_status_t sat_chain_destroy(sat_chain_t chain) {
     return SAT_OK;
 }
 
+// Tile order of a chained strip with R tile rows: anti-diagonal over groups of g vertically adjacent tiles
+// (order 3, tile_of_serial), g the largest of 8, 4, 2 dividing R: the strip's bottom tile of column J
+// resolves R/g group diagonals after its top tile -- the chain's lag per rank, (R/g) / (R/g + C) of a
+// strip -- and a column look-back (8 predecessors per poll round) spans the g - 1 tiles above in the group
+// plus the inclusive word of the group above.  SAT_CHAIN_ORDER overrides it (tuning: 2 = column-major).
+int chain_order(int R) {
+    if (const char* e = std::getenv("SAT_CHAIN_ORDER")) return std::atoi(e);
+    for (int g : {8, 4, 2})
+        if (R % g == 0) return 3 | (g << 8);
+    return 3;
+}
+
 SAT_API sat_status_t sat_compute_chained(sat_chain_t chain, sat_dtype_t dtype, const void* strip_src, void* strip_dst,
                                          int64_t strip_rows, int64_t cols, int64_t pitch, void* stream) {
     if (!chain) return fail(SAT_ERR_INVALID_VALUE, "null chain");
@@ -1323,15 +1339,21 @@ SAT_API sat_status_t sat_compute_chained(sat_chain_t chain, sat_dtype_t dtype, c
         if (!chain->peer[g]) return fail(SAT_ERR_INVALID_VALUE, "chain not connected (rank %d)", g);
     if (chain->calls + 2 >= sat::kEpochMax) return fail(SAT_ERR_UNSUPPORTED, "chain epoch exhausted: recreate it");
     Plan pl;
-    if ((s = make_plan(strip_rows, cols, pitch, strip_src, strip_dst, &pl, false, 0, kVarChain)) != SAT_OK) return s;
-    const Variant& v = variants()[kVarChain];
+    int cvi = kVarChain;
+    {
+        std::lock_guard<std::mutex> g(g_mu);
+        if (g_variant >= 0 && g_variant < static_cast<int>(variants().size()) && variants()[g_variant].chain)
+            cvi = g_variant;  // tuning hook: another chained configuration
+    }
+    if ((s = make_plan(strip_rows, cols, pitch, strip_src, strip_dst, &pl, false, 0, cvi)) != SAT_OK) return s;
+    const Variant& v = variants()[cvi];
     int dev = 0;
     SAT_CUDA(cudaGetDevice(&dev));
     if (dev != chain->dev) return fail(SAT_ERR_INVALID_VALUE, "chain lives on device %d, current device %d", chain->dev, dev);
     int occ = 0, sms = 0, max_ctas = 0;
     {
         std::lock_guard<std::mutex> g(g_mu);
-        if ((s = occupancy(dev, kVarChain, dtype, pl.tma, false, &occ)) != SAT_OK) return s;
+        if ((s = occupancy(dev, cvi, dtype, pl.tma, false, &occ)) != SAT_OK) return s;
         DeviceInfo* di = nullptr;
         if ((s = device_info(dev, &di)) != SAT_OK) return s;
         sms = di->sms;
@@ -1373,7 +1395,7 @@ SAT_API sat_status_t sat_compute_chained(sat_chain_t chain, sat_dtype_t dtype, c
     p.R = pl.R;
     p.C = pl.C;
     p.ntiles = static_cast<int>(pl.ntiles);
-    p.order = 2;
+    p.order = chain_order(pl.R);
     p.row_slots = chain->slots;
     p.col_slots = chain->slots + static_cast<size_t>(pl.ntiles) * v.TR;
     p.corner_slots = chain->slots + static_cast<size_t>(pl.ntiles) * (v.TR + v.TC);
@@ -1436,7 +1458,7 @@ SAT_API sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm) {
 #if SAT_STATS
     if (order < 0 || (order & 15) > 1 || order > 0xffff) return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
 #else
-    if (order < 0 || (order & ~0xff0f) != 0 || (order & 15) > 2)
+    if (order < 0 || (order & ~0xff0f) != 0 || (order & 15) > 3)
         return fail(SAT_ERR_INVALID_VALUE, "unknown order %d", order);
 #endif
     if (ctas_per_sm < 0) return fail(SAT_ERR_INVALID_VALUE, "ctas_per_sm < 0");
@@ -1456,6 +1478,18 @@ SAT_API sat_status_t sat_set_max_ctas(int max_ctas) {
 
 SAT_API int sat_num_variants(void) { return static_cast<int>(variants().size()); }
 
+SAT_API sat_status_t sat_debug_occupy(int ctas, int64_t ns, int64_t smem_bytes, void* stream) {
+    if (ctas < 1 || ns < 0 || ns > 10000000000LL || smem_bytes < 0 || smem_bytes > 227 * 1024)
+        return fail(SAT_ERR_INVALID_VALUE, "bad occupy arguments");
+    const int smem = static_cast<int>(smem_bytes);
+    SAT_CUDA(cudaFuncSetAttribute(reinterpret_cast<const void*>(&sat::occupy_kernel),
+                                  cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+    sat::occupy_kernel<<<ctas, 32, smem, static_cast<cudaStream_t>(stream)>>>(static_cast<long long>(ns));
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "occupy_kernel");
+    return SAT_OK;
+}
+
 SAT_API sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* tile_cols) {
     if (variant < 0 || variant >= static_cast<int>(variants().size()))
         return fail(SAT_ERR_INVALID_VALUE, "unknown variant %d", variant);
@@ -1466,7 +1500,7 @@ SAT_API sat_status_t sat_variant_info(int variant, int32_t* tile_rows, int32_t* 
 
 SAT_API sat_status_t sat_debug_tile_order(int64_t R, int64_t C, int order, int32_t* out, void* stream) {
     if (R <= 0 || C <= 0 || R * C > (int64_t(1) << 30) || !out || order < 0 || (order & ~0xff0f) != 0 ||
-        (order & 15) > 2)
+        (order & 15) > 3)
         return fail(SAT_ERR_INVALID_VALUE, "bad args");
     const int64_t n = R * C;
     int blocks = static_cast<int>((n + 255) / 256);

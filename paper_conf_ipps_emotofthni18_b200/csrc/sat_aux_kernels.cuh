@@ -122,4 +122,14 @@ __global__ void __launch_bounds__(1024) carry_prefix_kernel(const V* __restrict_
     }
 }
 
+// Test hook (sat_debug_occupy): each CTA holds `smem` bytes of shared memory and spins for `ns`
+// nanoseconds, so that a SAT launched next on another stream finds most SMs taken -- its persistent CTAs
+// then start over a long interval (forward progress under any CTA -> SM assignment).
+__global__ void occupy_kernel(long long ns) {
+    extern __shared__ unsigned char occ_smem[];
+    const uint64_t t0 = sat_now_ns();
+    if (threadIdx.x == 0) occ_smem[0] = 0;
+    while (sat_now_ns() - t0 < static_cast<uint64_t>(ns)) __nanosleep(1000);
+}
+
 }  // namespace sat

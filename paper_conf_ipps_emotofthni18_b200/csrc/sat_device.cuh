@@ -3,6 +3,7 @@
 #pragma once
 
 #include <cstdint>
+#include <cstdio>
 #include <cuda.h>  // CUtensorMap (header only; the driver entry point is resolved at run time)
 #include <cuda_runtime.h>
 
@@ -78,6 +79,59 @@ __device__ __forceinline__ V warp_sum(V x) {
     return x;
 }
 
+// ------------------------------------------------------------------ protocol-stress builds
+// (PAPER.md:21 -- the method must be correct and deadlock-free under any CTA -> SM
+// assignment and any relative speed of the CTAs.)  Neither switch is on in the product build.
+//   -DSAT_JITTER=1    every status-word / flag publication first sleeps a pseudo-random 0 .. 4 us (one
+//                     publication in four), so words land in orders the production timing never shows.
+//   -DSAT_WATCHDOG=1  every spin loop is bounded: after kWatchdogNs of waiting without progress the
+//                     thread prints what it waited for and traps, so a protocol deadlock becomes a launch
+//                     error (cudaErrorLaunchFailure) instead of a hung GPU.
+__device__ __forceinline__ uint64_t sat_now_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+#if SAT_JITTER
+__device__ __forceinline__ void sat_jitter() {
+    uint64_t z = static_cast<uint64_t>(clock64()) ^ (static_cast<uint64_t>(blockIdx.x) << 40) ^
+                 (static_cast<uint64_t>(threadIdx.x) << 20);
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
+    z ^= z >> 31;
+    if ((z & 3u) == 0u) __nanosleep(static_cast<unsigned>((z >> 8) & 4095u));
+}
+#else
+__device__ __forceinline__ void sat_jitter() {}
+#endif
+#if SAT_WATCHDOG
+constexpr uint64_t kWatchdogNs = 10000000000ull;  // 10 s without progress
+__device__ __noinline__ void sat_watchdog_fire(const char* what) {
+    printf("libsat watchdog: block %d thread %d waited > 10 s for %s\n", static_cast<int>(blockIdx.x),
+           static_cast<int>(threadIdx.x), what);
+    __trap();
+}
+#define SAT_SPIN_DECL uint64_t sat_spin_t0_ = ::sat::sat_now_ns()
+#define SAT_SPIN_RESET (sat_spin_t0_ = ::sat::sat_now_ns())
+#define SAT_SPIN_CHECK(what)                                                                                  \
+    do {                                                                                                      \
+        if (::sat::sat_now_ns() - sat_spin_t0_ > ::sat::kWatchdogNs) ::sat::sat_watchdog_fire(what);          \
+    } while (0)
+#else
+#define SAT_SPIN_DECL (void)0
+#define SAT_SPIN_RESET (void)0
+#define SAT_SPIN_CHECK(what) (void)0
+#endif
+// spin (with a nanosleep back-off) until `cond` holds
+#define sat_spin_until(cond, ns)                                                                              \
+    do {                                                                                                      \
+        SAT_SPIN_DECL;                                                                                        \
+        while (!(cond)) {                                                                                     \
+            SAT_SPIN_CHECK(#cond);                                                                            \
+            __nanosleep(ns);                                                                                  \
+        }                                                                                                     \
+    } while (0)
+
 // ------------------------------------------------------------------ shared memory / mbarrier
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -98,7 +152,23 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 
 // Blocking wait on an mbarrier phase.  The suspend-time hint lets the hardware park the warp until
 // the phase completes instead of spinning (a spinning warp steals issue slots from working warps).
+__device__ __forceinline__ bool mbar_try_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+        "selp.u32 %0, 1, 0, p;\n}"
+        : "=r"(ok)
+        : "r"(smem_addr(bar)), "r"(parity), "r"(1000000u)
+        : "memory");
+    return ok != 0u;
+}
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+#if SAT_WATCHDOG
+    SAT_SPIN_DECL;
+    while (!mbar_try_wait(bar, parity)) SAT_SPIN_CHECK("an mbarrier phase");
+    return;
+#endif
     asm volatile(
         "{\n\t.reg .pred p;\n"
         "SAT_WAIT_%=:\n\t"
@@ -186,9 +256,11 @@ __device__ __forceinline__ void prefetch_tensormap(const CUtensorMap* map) {
 // 64-bit access is single-copy atomic, so value and status can never tear; relaxed gpu-scope
 // accesses go to L2 (coherent point for all SMs) and need no fence (R11).
 __device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t a) {
+    sat_jitter();
     asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(a) : "memory");
 }
 __device__ __forceinline__ void st_relaxed2(uint64_t* p, uint64_t a, uint64_t b) {
+    sat_jitter();
     asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
 __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
@@ -203,9 +275,11 @@ __device__ __forceinline__ void ld_relaxed2(const uint64_t* p, uint64_t& a, uint
 // Status-word accesses with an L2 evict_last policy: the words must survive in L2 between their
 // publication and their successors' look-backs while the matrix streams through.
 __device__ __forceinline__ void st_relaxed_p(uint64_t* p, uint64_t a, uint64_t pol) {
+    sat_jitter();
     asm volatile("st.relaxed.gpu.global.L2::cache_hint.b64 [%0], %1, %2;" ::"l"(p), "l"(a), "l"(pol) : "memory");
 }
 __device__ __forceinline__ void st_relaxed2_p(uint64_t* p, uint64_t a, uint64_t b, uint64_t pol) {
+    sat_jitter();
     asm volatile("st.relaxed.gpu.global.L2::cache_hint.v2.b64 [%0], {%1, %2}, %3;" ::"l"(p), "l"(a), "l"(b), "l"(pol)
                  : "memory");
 }
@@ -224,12 +298,14 @@ __device__ __forceinline__ void ld_relaxed2_p(const uint64_t* p, uint64_t& a, ui
 // System-scope status words: the chained strip partition's inbox, written by a peer GPU over NVLink
 // (peer-mapped pointers) and polled by the owner; single-copy atomic 64-bit accesses as above.
 __device__ __forceinline__ void st_relaxed2_sys(uint64_t* p, uint64_t a, uint64_t b) {
+    sat_jitter();
     asm volatile("st.relaxed.sys.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
 __device__ __forceinline__ void ld_relaxed2_sys(const uint64_t* p, uint64_t& a, uint64_t& b) {
     asm volatile("ld.relaxed.sys.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
 __device__ __forceinline__ void st_relaxed_sys_u32(uint32_t* p, uint32_t a) {
+    sat_jitter();
     asm volatile("st.relaxed.sys.global.b32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
 }
 __device__ __forceinline__ uint32_t ld_relaxed_sys_u32(const uint32_t* p) {

@@ -64,16 +64,17 @@ struct Ctrl {
 };
 
 // Chained strip partition (sat_compute_chained): rank r's
-// strip takes its column carry from the strip column sums of every rank g < r, which rank g pushes
-// (as epoch-tagged status words, prefix form over each tile's columns) into rank r's inbox over
-// NVLink peer memory as soon as its bottom tile of that tile column resolves.
+// strip takes its column carry T(r-1) = the column sums of all rows of ranks 0 .. r-1, which rank r-1
+// pushes (as epoch-tagged status words, prefix form over each tile's columns) into rank r's inbox over
+// NVLink peer memory as soon as its bottom tile of that tile column resolves (T(r-1) = its own strip
+// column sums + the T(r-2) it received).
 constexpr int kMaxChainRanks = 8;
 struct ChainParams {
     int rank, nranks;
     uint32_t parity;                         // inbox half of this call (epoch & 1)
     int64_t inbox_cols;                      // words per inbox vector (>= C * TC)
-    uint64_t* peer_inbox[kMaxChainRanks];    // inbox of every rank: [2][kMaxChainRanks][inbox_cols] words
-    uint32_t* peer_done[kMaxChainRanks];     // back-pressure words of every rank: [kMaxChainRanks]
+    uint64_t* peer_inbox[kMaxChainRanks];    // inbox of every rank: [2][inbox_cols] words (written by rank - 1)
+    uint32_t* peer_done[kMaxChainRanks];     // back-pressure words of every rank: [kMaxChainRanks] (rank + 1's used)
 };
 
 template <typename V>
@@ -145,7 +146,10 @@ __device__ __forceinline__ void diag_of_serial(long long s, int R, int C, int& I
 // == 0 and g | C: anti-diagonal order of g-wide tile groups, the g tiles of a group consecutive and
 // left to right (a topological order too: a tile's left neighbour is earlier in its group or on the
 // previous group diagonal, its upper neighbours on the previous group diagonal).  The g tiles of a
-// group share their DRAM rows, so the rows concurrent tiles touch are g times longer.
+// group share their DRAM rows, so the rows concurrent tiles touch are g times longer.  order & 15 == 3
+// with g | R: anti-diagonal order of g-TALL tile groups, the g tiles of a group consecutive and top to
+// bottom (chained strips: the bottom tile of tile column J resolves R/g group diagonals after the top one,
+// and a column look-back spans at most the g - 1 tiles above in the group plus one inclusive word).
 __device__ __forceinline__ void tile_of_serial(int s_, int R, int C, int order, int& I, int& J) {
     if ((order & 15) == 1) {
         I = s_ / C;
@@ -158,6 +162,15 @@ __device__ __forceinline__ void tile_of_serial(int s_, int R, int C, int order, 
         return;
     }
     const int g = (order >> 8) & 255;
+    if ((order & 15) == 3) {
+        if (g > 1 && R % g == 0) {
+            diag_of_serial(s_ / g, R / g, C, I, J);
+            I = I * g + s_ % g;
+        } else {
+            diag_of_serial(s_, R, C, I, J);
+        }
+        return;
+    }
     if (g > 1 && C % g == 0) {
         int J2;
         diag_of_serial(s_ / g, R, C / g, I, J2);
@@ -180,6 +193,7 @@ __device__ __forceinline__ void lookback_vec(const uint64_t* p, long long step, 
     uint32_t pending = (1u << E) - 1u;
 #pragma unroll
     for (int e = 0; e < E; ++e) acc[e] = V(0);
+    SAT_SPIN_DECL;
     while (true) {
         if (pending) {
             ++steps;
@@ -190,6 +204,7 @@ __device__ __forceinline__ void lookback_vec(const uint64_t* p, long long step, 
                     if (((pending >> e) & 1u) && !word_ready(w[e], epoch)) ok = false;
                 if (ok) break;
                 ++spins;
+                SAT_SPIN_CHECK("a row / column look-back word");
                 __nanosleep(20);
                 ld_words<E>(p, w);
             }
@@ -224,6 +239,7 @@ __device__ __forceinline__ bool lookback_diag(const uint64_t* corner_slots, int 
     }
     V acc = V(0);
     int base = 1;
+    SAT_SPIN_DECL;
     while (true) {
         const int k = base + lane;
         const bool inrange = (I - k >= 0) && (J - k >= 0);
@@ -234,6 +250,7 @@ __device__ __forceinline__ bool lookback_diag(const uint64_t* corner_slots, int 
         const unsigned need = (f >= 31) ? kFull : ((2u << f) - 1u);
         if (notready & need) {
             if (!blocking) return false;
+            SAT_SPIN_CHECK("a diagonal look-back word");
             __nanosleep(20);
             w = diag_word(corner_slots, I, J, C, k);
             continue;

@@ -78,8 +78,11 @@ struct Slot {
 // stop.  Returns false when tile k will never exist.
 template <typename SM>
 __device__ __forceinline__ bool wait_acquired(SM& sm, int s, uint32_t parity, int k) {
-    while (!mbar_try(&sm.acq[s], parity))
+    SAT_SPIN_DECL;
+    while (!mbar_try(&sm.acq[s], parity)) {
         if (k >= *reinterpret_cast<volatile int*>(&sm.end_n)) return false;
+        SAT_SPIN_CHECK("a tile acquisition");
+    }
     return true;
 }
 
@@ -99,9 +102,9 @@ __device__ __forceinline__ void ws_exit(const KParams<V>& p, uint32_t epoch) {
         p.ctrl->exit_count = 0u;
         if (p.epoch_override == 0u) p.ctrl->epoch = (epoch >= kEpochMax) ? 1u : epoch + 1u;
         __threadfence();
-        // chained strips: every CTA of this rank is done reading its inbox for this call; tell the
-        // upstream ranks, which may then reuse this parity of the inbox two calls later
-        for (int g = 0; g < p.chain.rank; ++g) st_relaxed_sys_u32(p.chain.peer_done[g] + p.chain.rank, epoch);
+        // chained strips: every CTA of this rank is done reading its inbox for this call; tell the rank
+        // above (the only writer of this inbox), which may then reuse this parity two calls later
+        if (p.chain.rank > 0) st_relaxed_sys_u32(p.chain.peer_done[p.chain.rank - 1] + p.chain.rank, epoch);
     }
 }
 

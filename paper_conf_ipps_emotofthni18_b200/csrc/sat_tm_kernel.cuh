@@ -682,73 +682,61 @@ __device__ __forceinline__ bool lb_consume_n(uint32_t& pending, int& pos, V (&ac
 // resolved (acc = prefix_j of the column sums of this strip's rows above the tile, VP):
 //  1. the strip-local inclusive column words VP + LCS(I,J) (Step 2.B.3 within the strip), once the owning
 //     compute warp has written its local column aggregates;
-//  2. bottom tile row: those words are this strip's column sums over tile column J -- pushed into the
-//     inbox of every downstream rank (system-scope stores to peer memory), after the downstream ranks
-//     have released this inbox half (back-pressure: they finished call epoch - 2);
-//  3. acc += the strip column sums of every upstream rank g < rank from this rank's inbox (ascending g,
-//     so fp32 sums are associated the same way on every rank): acc = prefix_j GCS(I-1,J) of the full
-//     matrix, the column carry of Step 4 (the virtual tile row above the strip, R12).
+//  2. acc += the carry T(rank-1) of the rank above from this rank's inbox: acc = prefix_j GCS(I-1,J) of the
+//     full matrix, the column carry of Step 4 (the virtual tile row above the strip, R12);
+//  3. bottom tile row: LCS(I,J) + acc = T(rank), the column sums of every row of ranks 0..rank over tile
+//     column J (prefix form) -- pushed into the inbox of rank + 1 only (system-scope stores to peer
+//     memory), after rank + 1 has released this inbox half (back-pressure: it finished call epoch - 2).
+// The carry is forwarded cumulatively, T(r) = LCS + (VP + T(r-1)): every rank polls one vector and pushes
+// one, whatever N (reading R12': fp32 carries are associated rank by rank, top to bottom).  The push
+// of tile column J waits for T(rank-1)[J], which the top tile of column J needed already, so the chain
+// lags one tile column per rank.
 template <typename V, typename Cfg, typename SM>
 __device__ __forceinline__ void tm_chain_column(SM& sm, const KParams<V>& p, int s, int k, int I, int J,
                                                 V (&acc)[Cfg::EC], uint64_t* own, uint32_t epoch, int lane, bool& bp_ok) {
     constexpr int E = Cfg::EC, NW = Cfg::NW, TC = Cfg::TC;
     const uint64_t pol = policy_evict_last();
     const ChainParams& ch = p.chain;
-    while (*reinterpret_cast<const volatile int*>(&sm.lw[s][NW - 1]) != k + 1) __nanosleep(20);
+    sat_spin_until(*reinterpret_cast<const volatile int*>(&sm.lw[s][NW - 1]) == k + 1, 20);
     __threadfence_block();
-    uint64_t wv[E];
+    V lcs[E];
 #pragma unroll
-    for (int e = 0; e < E; ++e) wv[e] = pack(epoch, kIncl, to_bits(sm.lcs[s][lane * E + e] + acc[e]));
-    if (I > 0) st_words_p<E>(own + lane * E, wv, pol);  // I == 0: published inclusive by the compute warp
+    for (int e = 0; e < E; ++e) lcs[e] = sm.lcs[s][lane * E + e];
+    if (I > 0) {  // I == 0: published inclusive by the compute warp
+        uint64_t wv[E];
+#pragma unroll
+        for (int e = 0; e < E; ++e) wv[e] = pack(epoch, kIncl, to_bits(lcs[e] + acc[e]));
+        st_words_p<E>(own + lane * E, wv, pol);
+    }
     const long long col = static_cast<long long>(J) * TC + lane * E;
+    if (ch.rank > 0) {
+        const uint64_t* inbox = ch.peer_inbox[ch.rank] + static_cast<long long>(ch.parity) * ch.inbox_cols + col;
+        uint64_t w[E];
+        SAT_SPIN_DECL;
+        while (true) {
+            ld_words_sys<E>(inbox, w);
+            bool ok = true;
+#pragma unroll
+            for (int e = 0; e < E; ++e) ok = ok && word_ready(w[e], epoch);
+            if (__all_sync(kFull, ok)) break;
+            SAT_SPIN_CHECK("chain inbox");
+            __nanosleep(64);
+        }
+#pragma unroll
+        for (int e = 0; e < E; ++e) acc[e] = acc[e] + from_bits<V>(static_cast<uint32_t>(w[e]));
+    }
     if (I == p.R - 1 && ch.rank + 1 < ch.nranks) {
         if (!bp_ok) {
-            for (int r = ch.rank + 1 + lane; r < ch.nranks; r += 32)
-                while (static_cast<long long>(ld_relaxed_sys_u32(ch.peer_done[ch.rank] + r)) <
-                       static_cast<long long>(epoch) - 2)
-                    __nanosleep(64);
+            if (lane == 0)
+                sat_spin_until(static_cast<long long>(ld_relaxed_sys_u32(ch.peer_done[ch.rank] + ch.rank + 1)) >=
+                                   static_cast<long long>(epoch) - 2, 64);
             __syncwarp();
             bp_ok = true;
         }
-        for (int r = ch.rank + 1; r < ch.nranks; ++r)
-            st_words_sys<E>(ch.peer_inbox[r] + (static_cast<long long>(ch.parity) * kMaxChainRanks + ch.rank) *
-                                                   ch.inbox_cols + col, wv);
-    }
-    if (ch.rank > 0) {
-        const uint64_t* inbox = ch.peer_inbox[ch.rank] + static_cast<long long>(ch.parity) * kMaxChainRanks * ch.inbox_cols + col;
-        // upstream ranks in groups of 4: each poll round loads every vector of the group still missing;
-        // a group is added (in ascending g) once all of it is in
-        for (int g0 = 0; g0 < ch.rank; g0 += 4) {
-            const int ng = ch.rank - g0 < 4 ? ch.rank - g0 : 4;
-            uint32_t pend = (1u << ng) - 1u;
-            V part[4][E];
-            while (true) {
-                uint64_t w[4][E];
+        uint64_t wv[E];
 #pragma unroll
-                for (int h = 0; h < 4; ++h)
-                    if ((pend >> h) & 1u) ld_words_sys<E>(inbox + static_cast<long long>(g0 + h) * ch.inbox_cols, w[h]);
-#pragma unroll
-                for (int h = 0; h < 4; ++h) {
-                    if ((pend >> h) & 1u) {
-                        bool ok = true;
-#pragma unroll
-                        for (int e = 0; e < E; ++e) ok = ok && word_ready(w[h][e], epoch);
-                        if (__all_sync(kFull, ok)) {
-#pragma unroll
-                            for (int e = 0; e < E; ++e) part[h][e] = from_bits<V>(static_cast<uint32_t>(w[h][e]));
-                            pend &= ~(1u << h);
-                        }
-                    }
-                }
-                if (!pend) break;
-                __nanosleep(64);
-            }
-#pragma unroll
-            for (int h = 0; h < 4; ++h)
-                if (h < ng)
-#pragma unroll
-                    for (int e = 0; e < E; ++e) acc[e] = acc[e] + part[h][e];
-        }
+        for (int e = 0; e < E; ++e) wv[e] = pack(epoch, kIncl, to_bits(lcs[e] + acc[e]));
+        st_words_sys<E>(ch.peer_inbox[ch.rank + 1] + static_cast<long long>(ch.parity) * ch.inbox_cols + col, wv);
     }
 }
 
@@ -802,6 +790,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
         V dacc = V(0);
         int dbase = 1;
         bool cin = false, lpub = false;
+        SAT_SPIN_DECL;
         while (true) {
             // ---- issue this round's loads
             uint64_t w[NP][E], wd = 0;
@@ -877,7 +866,12 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                 lpub = __shfl_sync(kFull, go, 31) != 0;
             }
             if (cin && ddone) break;
-            if (!progress) __nanosleep(32);
+            if (progress) {
+                SAT_SPIN_RESET;
+            } else {
+                SAT_SPIN_CHECK(ROW ? "row / diagonal look-back words" : "column look-back words");
+                __nanosleep(32);
+            }
         }
         // ---- Step 3.3 (GS, by whoever comes last) and the hand-off
         if (ROW && Cfg::CHAIN) {
@@ -888,7 +882,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
             __threadfence_block();
             if (lane == 0) *reinterpret_cast<volatile int*>(&sm.rdone[s]) = k + 1;
             if (J > 0) {
-                while (flag(&sm.cdone[s]) != k + 1) __nanosleep(20);
+                sat_spin_until(flag(&sm.cdone[s]) == k + 1, 20);
                 __threadfence_block();
                 if (lane == 31) st_relaxed_p(p.corner_slots + tidx, pack(epoch, kIncl, to_bits(dacc + sm.cp[s][TC - 1])), pol);
             }
@@ -1068,13 +1062,14 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         Slot<Cfg::NQ> ta, tl;
         Slot<IN> sl;
         bool acq_done = false;
+        SAT_SPIN_DECL;
         while (true) {
             bool progress = false;
             if (!acq_done && (ta.k < Cfg::NQ || mbar_test(&sm.tfree[ta.s], ta.ph ^ 1u))) {
                 const int t = static_cast<int>(atomicAdd(&p.ctrl->counter, 1u));
                 const bool valid = t < p.ntiles;
                 TileInfo ti{t, 0, 0, 0};
-                if (valid) tile_of_serial(t, p.R, p.C, Cfg::CHAIN ? 2 : p.order, ti.I, ti.J);
+                if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
                 sm.info[ta.s] = ti;
                 if (!valid) {
                     *reinterpret_cast<volatile int*>(&sm.end_n) = ta.k;
@@ -1117,7 +1112,12 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 if (tl.k < ta.k) WS_ST(kWsLdEmptyWait, b1 - b0);                 // stage not yet read
             }
 #else
-            if (!progress) __nanosleep(32);
+            if (progress) {
+                SAT_SPIN_RESET;
+            } else {
+                SAT_SPIN_CHECK("a free tile slot or input stage (loader)");
+                __nanosleep(32);
+            }
 #endif
         }
     }

@@ -409,6 +409,27 @@ def test_device_grouped_tile_order_is_topological(sat, R, C, g):
     assert [tuple(t) for t in got[:g].tolist()] == [(0, j) for j in range(g)]
 
 
+@pytest.mark.parametrize("R,C,g", [(64, 512, 8), (16, 5, 4), (8, 3, 8), (6, 7, 2), (7, 9, 4), (1, 5, 2)])
+def test_device_tall_grouped_tile_order_is_topological(sat, R, C, g):
+    """Order 3 (chained strips): anti-diagonal order of g-tall groups, a group's tiles consecutive top to
+    bottom; a topological permutation of the R x C tiles; with g not dividing R the
+    plain Fig. 9 order."""
+    got = sat.debug_tile_order(R, C, 3 | (g << 8)).cpu().numpy()
+    if R % g:
+        assert (got == np.array(oracle.tile_order(R, C))).all()
+        return
+    assert sorted(map(tuple, got.tolist())) == [(I, J) for I in range(R) for J in range(C)]
+    pos = {tuple(t): k for k, t in enumerate(got.tolist())}
+    for (I, J), k in pos.items():
+        for dep in [(I, J - 1), (I - 1, J), (I - 1, J - 1)]:
+            if dep[0] >= 0 and dep[1] >= 0:
+                assert pos[dep] < k
+    assert [tuple(t) for t in got[:g].tolist()] == [(i, 0) for i in range(g)]
+    # the bottom tile of column J comes R/g group diagonals after the top one
+    for J in range(C):
+        assert pos[(R - 1, J)] - pos[(0, J)] < (R // g) * (R // g + 1) * g
+
+
 # ----------------------------------------------------------------------------------- full-size (BASELINE configs)
 def _streaming_check(sat, rows, cols, dist, seed, chunk=2048):
     """Full-size parity in the launch configuration bench.py times: device-generated input, one SAT
