@@ -88,6 +88,33 @@ sat_status_t sat_compute_f32(const float* src, float* dst, int64_t rows, int64_t
 sat_status_t sat_compute_u8(const uint8_t* src, int64_t src_pitch, uint32_t* dst, int64_t rows,
                             int64_t cols, int64_t pitch, void* stream);
 
+/* fp32 input, fp64 SAT (the accumulation the paper's 4-byte float, P:253,
+ * cannot hold exactly at large n).  dst[i][j] = sum of src[0..i][0..j], every addition in IEEE
+ * fp64 (round to nearest); the fp32 -> fp64 widening is exact.  Same single-pass look-back method
+ * (Sec. IV) with each 64-bit aggregate published as two tagged status words; one CTA per
+ * 64 x 128 tile.  4 B read + 8 B written per element.
+ *   src  device fp32, rows x cols, row stride src_pitch ELEMENTS (>= cols); read once.
+ *   dst  device fp64, rows x cols, row stride dst_pitch ELEMENTS (>= cols); must not overlap src;
+ *        pad elements are never written.
+ * Accuracy: |dst - exact| <= (rows + cols) * 2.3e-16 * SAT(|src|) at every entry (the R10 argument
+ * with the fp64 unit roundoff); exact while every partial sum is an integer < 2^53.  16-byte aligned
+ * pointers with src_pitch % 4 == 0 and dst_pitch % 2 == 0 take the vector path.
+ * Errors: INVALID_VALUE (sizes, overlap, NULL), MISALIGNED (src not 4-byte or dst not 8-byte
+ * aligned), UNSUPPORTED (rows or cols >= 2^31), OUT_OF_MEMORY (workspace), CUDA.  Stream-ordered. */
+sat_status_t sat_compute_f32_f64(const float* src, int64_t src_pitch, double* dst, int64_t dst_pitch,
+                                 int64_t rows, int64_t cols, void* stream);
+
+/* Moments for summed-area variance shadow maps (Lauritzen, ref. [8] at P:311): the SAT of a and
+ * the SAT of a*a, in fp32, interleaved: dst[2*(i*dst_pitch + j)] = SAT(a)[i][j],
+ * dst[2*(i*dst_pitch + j) + 1] = SAT(a*a)[i][j] (a*a rounded to fp32 once, then summed like
+ * sat_compute_f32).  Same method and kernel as sat_compute_f32_f64 (the pair is one 64-bit element).
+ *   src  device fp32, row stride src_pitch ELEMENTS (>= cols).
+ *   dst  device fp32 pairs, row stride dst_pitch PAIRS (>= cols); must not overlap src.
+ * Accuracy: each channel within (rows + cols) * 1.2e-7 * its absSAT (SAT(|a|), resp. SAT(a*a)).
+ * Errors: as sat_compute_f32_f64. */
+sat_status_t sat_compute_moments_f32(const float* src, int64_t src_pitch, float* dst, int64_t dst_pitch,
+                                     int64_t rows, int64_t cols, void* stream);
+
 /* Same as above for either dtype, plus an optional carry row.
  *   carry  device, `cols` elements of the same dtype, or NULL.  When given, carry[j] is added to
  *          every element of column j of the result: dst[i][j] = carry[j] + SAT(src)[i][j].  With

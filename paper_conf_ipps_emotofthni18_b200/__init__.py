@@ -21,7 +21,7 @@ from ._lib import SAT_FLOAT32, SAT_INT32, SatError, SatPlan, check
 _lib.lib()  # load now: fail loudly at import if the native library is missing
 
 __all__ = [
-    "sat", "sat_batched", "sat_batched_u8", "sat_u8", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
+    "sat", "sat_batched", "sat_batched_u8", "sat_u8", "sat_f64", "sat_moments", "sat_host", "compute", "box_sum", "rect_sums", "strip_colsum", "carry_prefix", "Comm", "sat_sharded", "strip_bounds",
     "Chain", "sat_chained", "exchange_blobs",
     "strip_layout", "broadcast_unique_id",
     "query_plan", "set_tuning", "set_max_ctas", "num_variants", "variant_info", "debug_tile_order", "debug_occupy", "debug_workspace",
@@ -171,6 +171,44 @@ def sat_u8(src, out=None, *, stream=None):
     with torch.cuda.device(src.device):
         check(_lib.lib().sat_compute_u8(src.data_ptr(), spitch, out.data_ptr(), rows, cols, opitch,
                                         _stream_ptr(stream)), "sat_compute_u8")
+    return out
+
+
+def sat_f64(src, out=None, *, stream=None):
+    """fp64 SAT of a 2-D float32 CUDA tensor (sat_compute_f32_f64, NEXT-3): returns float64 (rows, cols)."""
+    torch = _torch()
+    if src.dtype != torch.float32:
+        raise TypeError("sat_f64 needs a float32 tensor")
+    rows, cols, spitch = _matrix(src, "src")
+    if out is None:
+        out = torch.empty((rows, cols), dtype=torch.float64, device=src.device)
+    if out.dtype != torch.float64 or out.device != src.device:
+        raise ValueError("out must be a float64 tensor on src's device")
+    orows, ocols, opitch = _matrix(out, "out")
+    if (orows, ocols) != (rows, cols):
+        raise ValueError("out must have src's shape")
+    with torch.cuda.device(src.device):
+        check(_lib.lib().sat_compute_f32_f64(src.data_ptr(), spitch, out.data_ptr(), opitch, rows, cols,
+                                             _stream_ptr(stream)), "sat_compute_f32_f64")
+    return out
+
+
+def sat_moments(src, out=None, *, stream=None):
+    """Summed-area variance shadow map moments of a 2-D float32 CUDA tensor (sat_compute_moments_f32):
+    returns float32 (rows, cols, 2) with [..., 0] = SAT(a) and [..., 1] = SAT(a*a)."""
+    torch = _torch()
+    if src.dtype != torch.float32:
+        raise TypeError("sat_moments needs a float32 tensor")
+    rows, cols, spitch = _matrix(src, "src")
+    if out is None:
+        out = torch.empty((rows, cols, 2), dtype=torch.float32, device=src.device)
+    if out.dtype != torch.float32 or out.device != src.device or out.dim() != 3 or tuple(out.shape) != (rows, cols, 2) \
+            or out.stride(2) != 1 or out.stride(1) != 2 or (rows > 1 and out.stride(0) % 2):
+        raise ValueError("out must be a float32 (rows, cols, 2) tensor of contiguous pairs on src's device")
+    opitch = out.stride(0) // 2 if rows > 1 else cols
+    with torch.cuda.device(src.device):
+        check(_lib.lib().sat_compute_moments_f32(src.data_ptr(), spitch, out.data_ptr(), opitch, rows, cols,
+                                                 _stream_ptr(stream)), "sat_compute_moments_f32")
     return out
 
 

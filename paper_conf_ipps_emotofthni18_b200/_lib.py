@@ -22,7 +22,7 @@ STATUS_NAMES = {
 
 # every symbol declared in include/sat.h (checked by tests/test_abi.py against the header)
 EXPORTS = (
-    "sat_compute_i32", "sat_compute_f32", "sat_compute_u8", "sat_compute", "sat_compute_host", "sat_compute_batched", "sat_compute_batched_u8", "sat_box_sum", "sat_rect_sums",
+    "sat_compute_i32", "sat_compute_f32", "sat_compute_u8", "sat_compute_f32_f64", "sat_compute_moments_f32", "sat_compute", "sat_compute_host", "sat_compute_batched", "sat_compute_batched_u8", "sat_box_sum", "sat_rect_sums",
     "sat_strip_colsum",
     "sat_carry_prefix", "sat_comm_get_unique_id", "sat_comm_init", "sat_comm_destroy", "sat_compute_sharded",
     "sat_chain_create", "sat_chain_export", "sat_chain_connect", "sat_chain_connect_local", "sat_chain_destroy",
@@ -61,6 +61,8 @@ def _declare(lib):
         "sat_compute_f32": [_vp, _vp, _i64, _i64, _i64, _vp],
         "sat_compute": [_int, _vp, _vp, _i64, _i64, _i64, _vp, _vp],
         "sat_compute_u8": [_vp, _i64, _vp, _i64, _i64, _i64, _vp],
+        "sat_compute_f32_f64": [_vp, _i64, _vp, _i64, _i64, _i64, _vp],
+        "sat_compute_moments_f32": [_vp, _i64, _vp, _i64, _i64, _i64, _vp],
         "sat_compute_host": [_int, _vp, _vp, _i64, _i64, _i64, _vp],
         "sat_compute_batched": [_int, _vp, _vp, _i64, _i64, _i64, _i64, _i64, _vp],
         "sat_compute_batched_u8": [_vp, _i64, _i64, _vp, _i64, _i64, _i64, _i64, _i64, _vp],

@@ -22,6 +22,7 @@
 #include "sat_tm_kernel.cuh"
 #include "sat_query_kernels.cuh"
 #include "sat_batch_kernel.cuh"
+#include "sat_wide_kernel.cuh"
 
 #if defined(SAT_HAVE_NCCL_H)
 #include <nccl.h>
@@ -243,6 +244,7 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32>>(),     // 7
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 4>>(),      // 8
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 0, 32>>(),      // 9: flat, diagonal 32
+        make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),                // 10: flat, tile ring of 8
 #if SAT_EXPERIMENTAL
         make_variant<sat::TmCfg<16, 2, 5>>(),  // 5: walkers publish (blocking ws_walker)
         make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 6
@@ -285,6 +287,21 @@ int auto_variant(int64_t rows, int64_t cols) {
     // 64 x 256 tiles
     const int64_t n = rows * cols;
     return n <= (int64_t(1) << 21) ? kVarClassic : (n <= (int64_t(1) << 25) ? kVarTm128 : kVarFlat);
+}
+
+// L2 prefetch of a tile's boxes when the loader acquires it (cp.async.bulk.prefetch.tensor): the DRAM read
+// of a tile then starts up to NQ - IN tiles before an input stage is free for it, so the read stream no
+// longer waits on the compute warps' stage release.  Measured on the flat 64 x 256 kernel at 32K^2
+// (tools/gpu_r02c.sh, profiles/r02_sweep_prefetch.jsonl): fp32 1.417 -> 1.384 ms, int32 1.409 -> 1.378 ms;
+// with a tile ring of 8 it over-fetches (1.50 ms).  It pays at every size (profiles/r02_sweep_prefetch_sizes.jsonl:
+// 4K^2 40.9 -> 36.7 us, 8K^2 108 -> 102 us, 64K^2 5.55 -> 5.48 ms).  Default: on for the TMEM-parked kernels
+// (the classic kernel has no tile ring); SAT_L2_PREFETCH=0/1 (read once) forces it off / on (tuning switch).
+int l2_prefetch_mode(int vi) {
+    static const int mode = [] {
+        const char* e = std::getenv("SAT_L2_PREFETCH");
+        return e ? std::atoi(e) : -1;
+    }();
+    return mode >= 0 ? mode : (variants()[vi].family == 2 ? 1 : 0);
 }
 
 int auto_order(int vi, int64_t cols) {
@@ -600,6 +617,10 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
     }
     int per_sm = (ctas_per_sm > 0 && ctas_per_sm < occ) ? ctas_per_sm : occ;
     int64_t grid = static_cast<int64_t>(sms) * per_sm;
+    // the classic kernel is launched the paper's way, one CTA per tile (CTAs beyond the resident
+    // ones take their tickets when they start, so any grid is deadlock-free): its persistent loop only
+    // runs under a CTA cap (sat_set_max_ctas, the forward-progress tests)
+    if (v.family == 0) grid = pl.ntiles;
     if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
     if (grid > pl.ntiles) grid = pl.ntiles;
 
@@ -645,6 +666,7 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
     p.src8 = u8 ? static_cast<const uint8_t*>(src) : nullptr;
     p.src_pitch = u8 ? src_pitch : pitch;
     if (u8) p.src = nullptr;
+    p.l2_prefetch = l2_prefetch_mode(pl.vi);
 #if SAT_STATS
     {
         std::lock_guard<std::mutex> lk(g_mu);
@@ -669,6 +691,57 @@ sat_status_t compute_impl(int dt, const void* src, void* dst, int64_t rows, int6
     w->last_TC = v.TC;
     w->last_R = pl.R;
     w->last_C = pl.C;
+    return SAT_OK;
+}
+
+// 64-bit output elements: moments = false -> fp64 SAT of fp32 input, true ->
+// (SAT(a), SAT(a*a)) fp32 pairs.  One CTA per 64 x 128 tile (sat_wide_kernel.cuh).
+sat_status_t wide_impl(bool moments, const float* src, int64_t src_pitch, void* dst, int64_t dst_pitch, int64_t rows,
+                       int64_t cols, cudaStream_t st) {
+    if (rows < 0 || cols < 0 || src_pitch < cols || dst_pitch < cols)
+        return fail(SAT_ERR_INVALID_VALUE, "bad sizes rows=%lld cols=%lld src_pitch=%lld dst_pitch=%lld", (long long)rows,
+                    (long long)cols, (long long)src_pitch, (long long)dst_pitch);
+    if (rows == 0 || cols == 0) return SAT_OK;
+    if (!src || !dst) return fail(SAT_ERR_INVALID_VALUE, "null pointer");
+    const uintptr_t a = reinterpret_cast<uintptr_t>(src), b = reinterpret_cast<uintptr_t>(dst);
+    if ((a & 3u) || (b & 7u)) return fail(SAT_ERR_MISALIGNED, "src must be 4-byte and dst 8-byte aligned");
+    if (rows > (int64_t(1) << 31) - 1 || cols > (int64_t(1) << 31) - 1)
+        return fail(SAT_ERR_UNSUPPORTED, "rows and cols must be < 2^31");
+    const uintptr_t na = static_cast<uintptr_t>(((rows - 1) * src_pitch + cols) * 4);
+    const uintptr_t nb = static_cast<uintptr_t>(((rows - 1) * dst_pitch + cols) * 8);
+    if (a < b + nb && b < a + na) return fail(SAT_ERR_INVALID_VALUE, "src and dst overlap");
+    constexpr int TR = sat::kWideTR, TC = sat::kWideTC;
+    const int64_t R = (rows + TR - 1) / TR, C = (cols + TC - 1) / TC, ntiles = R * C;
+    if (ntiles > (int64_t(1) << 31) - 1) return fail(SAT_ERR_UNSUPPORTED, "too many tiles");
+    int dev = 0;
+    SAT_CUDA(cudaGetDevice(&dev));
+    Workspace* w;
+    sat_status_t s = find_workspace(dev, st, &w);
+    if (s != SAT_OK) return s;
+    std::lock_guard<std::mutex> wlk(w->mu);
+    if ((s = grow_slots(w, static_cast<size_t>(ntiles) * 2 * (TR + TC + 1))) != SAT_OK) return s;
+    sat::WideParams p;
+    std::memset(&p, 0, sizeof(p));
+    p.src = src;
+    p.dst = dst;
+    p.rows = rows;
+    p.cols = cols;
+    p.src_pitch = src_pitch;
+    p.dst_pitch = dst_pitch;
+    p.R = static_cast<int>(R);
+    p.C = static_cast<int>(C);
+    p.ntiles = static_cast<int>(ntiles);
+    p.row_slots = w->slots;
+    p.col_slots = w->slots + static_cast<size_t>(ntiles) * 2 * TR;
+    p.corner_slots = w->slots + static_cast<size_t>(ntiles) * 2 * (TR + TC);
+    p.ctrl = w->ctrl;
+    p.vec = ((a & 15u) == 0 && (b & 15u) == 0 && (src_pitch * 4) % 16 == 0 && (dst_pitch * 8) % 16 == 0) ? 1 : 0;
+    if (moments) sat::sat_wide_kernel<float2><<<static_cast<unsigned>(ntiles), sat::kWideNW * 32, 0, st>>>(p);
+    else sat::sat_wide_kernel<double><<<static_cast<unsigned>(ntiles), sat::kWideNW * 32, 0, st>>>(p);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "sat_wide_kernel launch");
+    w->calls++;
+    w->last_TR = w->last_TC = w->last_R = w->last_C = 0;  // two words per value: not sat_debug_workspace's layout
     return SAT_OK;
 }
 
@@ -997,6 +1070,16 @@ SAT_API sat_status_t sat_compute_f32(const float* src, float* dst, int64_t rows,
 SAT_API sat_status_t sat_compute_u8(const uint8_t* src, int64_t src_pitch, uint32_t* dst, int64_t rows, int64_t cols,
                                     int64_t pitch, void* stream) {
     return compute_impl(kU8, src, dst, rows, cols, pitch, nullptr, static_cast<cudaStream_t>(stream), src_pitch);
+}
+
+SAT_API sat_status_t sat_compute_f32_f64(const float* src, int64_t src_pitch, double* dst, int64_t dst_pitch,
+                                         int64_t rows, int64_t cols, void* stream) {
+    return wide_impl(false, src, src_pitch, dst, dst_pitch, rows, cols, static_cast<cudaStream_t>(stream));
+}
+
+SAT_API sat_status_t sat_compute_moments_f32(const float* src, int64_t src_pitch, float* dst, int64_t dst_pitch,
+                                             int64_t rows, int64_t cols, void* stream) {
+    return wide_impl(true, src, src_pitch, dst, dst_pitch, rows, cols, static_cast<cudaStream_t>(stream));
 }
 
 SAT_API sat_status_t sat_strip_colsum(sat_dtype_t dtype, const void* src, void* colsum, int64_t rows, int64_t cols,
@@ -1396,6 +1479,7 @@ SAT_API sat_status_t sat_compute_chained(sat_chain_t chain, sat_dtype_t dtype, c
     p.C = pl.C;
     p.ntiles = static_cast<int>(pl.ntiles);
     p.order = chain_order(pl.R);
+    p.l2_prefetch = l2_prefetch_mode(cvi);
     p.row_slots = chain->slots;
     p.col_slots = chain->slots + static_cast<size_t>(pl.ntiles) * v.TR;
     p.corner_slots = chain->slots + static_cast<size_t>(pl.ntiles) * (v.TR + v.TC);

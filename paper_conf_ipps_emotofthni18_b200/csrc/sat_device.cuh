@@ -82,8 +82,8 @@ __device__ __forceinline__ V warp_sum(V x) {
 // ------------------------------------------------------------------ protocol-stress builds
 // (PAPER.md:21 -- the method must be correct and deadlock-free under any CTA -> SM
 // assignment and any relative speed of the CTAs.)  Neither switch is on in the product build.
-//   -DSAT_JITTER=1    every status-word / flag publication first sleeps a pseudo-random 0 .. 4 us (one
-//                     publication in four), so words land in orders the production timing never shows.
+//   -DSAT_JITTER=1    before every publication of status words a warp sleeps a pseudo-random 0 .. 4 us
+//                     (one time in four), so words land in orders the production timing never shows.
 //   -DSAT_WATCHDOG=1  every spin loop is bounded: after kWatchdogNs of waiting without progress the
 //                     thread prints what it waited for and traps, so a protocol deadlock becomes a launch
 //                     error (cudaErrorLaunchFailure) instead of a hung GPU.
@@ -92,17 +92,22 @@ __device__ __forceinline__ uint64_t sat_now_ns() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+// Jitter is applied per warp at publication points where the whole warp is converged (SAT_JITTER_WARP()
+// in the kernels): the lanes of a warp sleep the same time, so the perturbation is between warps and CTAs
+// -- what the look-back protocol must tolerate -- not inside a warp's lock-step code.
 #if SAT_JITTER
-__device__ __forceinline__ void sat_jitter() {
+__device__ __forceinline__ void sat_jitter_warp() {
     uint64_t z = static_cast<uint64_t>(clock64()) ^ (static_cast<uint64_t>(blockIdx.x) << 40) ^
-                 (static_cast<uint64_t>(threadIdx.x) << 20);
+                 (static_cast<uint64_t>(threadIdx.x >> 5) << 20);
     z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ull;
     z = (z ^ (z >> 27)) * 0x94d049bb133111ebull;
     z ^= z >> 31;
+    z = __shfl_sync(0xffffffffu, z, 0);
     if ((z & 3u) == 0u) __nanosleep(static_cast<unsigned>((z >> 8) & 4095u));
 }
+#define SAT_JITTER_WARP() ::sat::sat_jitter_warp()
 #else
-__device__ __forceinline__ void sat_jitter() {}
+#define SAT_JITTER_WARP() (void)0
 #endif
 #if SAT_WATCHDOG
 constexpr uint64_t kWatchdogNs = 10000000000ull;  // 10 s without progress
@@ -256,11 +261,9 @@ __device__ __forceinline__ void prefetch_tensormap(const CUtensorMap* map) {
 // 64-bit access is single-copy atomic, so value and status can never tear; relaxed gpu-scope
 // accesses go to L2 (coherent point for all SMs) and need no fence (R11).
 __device__ __forceinline__ void st_relaxed(uint64_t* p, uint64_t a) {
-    sat_jitter();
     asm volatile("st.relaxed.gpu.global.b64 [%0], %1;" ::"l"(p), "l"(a) : "memory");
 }
 __device__ __forceinline__ void st_relaxed2(uint64_t* p, uint64_t a, uint64_t b) {
-    sat_jitter();
     asm volatile("st.relaxed.gpu.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
 __device__ __forceinline__ uint64_t ld_relaxed(const uint64_t* p) {
@@ -275,11 +278,9 @@ __device__ __forceinline__ void ld_relaxed2(const uint64_t* p, uint64_t& a, uint
 // Status-word accesses with an L2 evict_last policy: the words must survive in L2 between their
 // publication and their successors' look-backs while the matrix streams through.
 __device__ __forceinline__ void st_relaxed_p(uint64_t* p, uint64_t a, uint64_t pol) {
-    sat_jitter();
     asm volatile("st.relaxed.gpu.global.L2::cache_hint.b64 [%0], %1, %2;" ::"l"(p), "l"(a), "l"(pol) : "memory");
 }
 __device__ __forceinline__ void st_relaxed2_p(uint64_t* p, uint64_t a, uint64_t b, uint64_t pol) {
-    sat_jitter();
     asm volatile("st.relaxed.gpu.global.L2::cache_hint.v2.b64 [%0], {%1, %2}, %3;" ::"l"(p), "l"(a), "l"(b), "l"(pol)
                  : "memory");
 }
@@ -298,14 +299,12 @@ __device__ __forceinline__ void ld_relaxed2_p(const uint64_t* p, uint64_t& a, ui
 // System-scope status words: the chained strip partition's inbox, written by a peer GPU over NVLink
 // (peer-mapped pointers) and polled by the owner; single-copy atomic 64-bit accesses as above.
 __device__ __forceinline__ void st_relaxed2_sys(uint64_t* p, uint64_t a, uint64_t b) {
-    sat_jitter();
     asm volatile("st.relaxed.sys.global.v2.b64 [%0], {%1, %2};" ::"l"(p), "l"(a), "l"(b) : "memory");
 }
 __device__ __forceinline__ void ld_relaxed2_sys(const uint64_t* p, uint64_t& a, uint64_t& b) {
     asm volatile("ld.relaxed.sys.global.v2.b64 {%0, %1}, [%2];" : "=l"(a), "=l"(b) : "l"(p) : "memory");
 }
 __device__ __forceinline__ void st_relaxed_sys_u32(uint32_t* p, uint32_t a) {
-    sat_jitter();
     asm volatile("st.relaxed.sys.global.b32 [%0], %1;" ::"l"(p), "r"(a) : "memory");
 }
 __device__ __forceinline__ uint32_t ld_relaxed_sys_u32(const uint32_t* p) {

@@ -95,6 +95,7 @@ struct KParams {
     const uint8_t* src8;  // u8 input (integral images, sat_compute_u8): generic path only, else nullptr
     int64_t src_pitch;    // row stride of src8 in bytes
     uint32_t epoch_override;  // != 0: the launch epoch chosen by the host (chained calls); ctrl->epoch untouched
+    int l2_prefetch;          // TMEM-parked kernels: L2 prefetch of a tile's boxes as soon as it is acquired
     ChainParams chain;        // chained strip partition only
 };
 
@@ -464,6 +465,7 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
                 for (int c = 0; c < 4; ++c) v[r][c] = v[r][c] + off[c];
         }
 
+        SAT_JITTER_WARP();
         // ---- Steps 2.A.1 / 2.B.1: publish the local aggregates straight from the owning lanes.
         //      Row slots: lane 31 of every warp (last column of its rows); column slots: the last
         //      warp (bottom row).  Edge tiles publish inclusive at once (their carry is zero).
@@ -530,6 +532,7 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
         SAT_CLK(c_b3b);
         if (warp == 3) SAT_ST(kStBar3Producer, c_b3b - c_b3a); else SAT_ST(kStBar3, c_b3b - c_b3a);
 
+        SAT_JITTER_WARP();
         // ---- Steps 2.A.3 / 2.B.3: publish the inclusive aggregates (owners of the local values)
         if (lane == 31 && J > 0) {
             uint64_t* rs = p.row_slots + tidx * TR + row0;

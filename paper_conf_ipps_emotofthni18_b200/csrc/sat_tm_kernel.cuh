@@ -413,6 +413,7 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
 #pragma unroll
             for (int x = 0; x < X; ++x) v[r][x] = v[r][x] + off[x];
     }
+    SAT_JITTER_WARP();
     // Steps 2.A.1 / 2.B.1 (edge tiles publish inclusive at once: their carry is zero)
     const uint64_t pol = policy_evict_last();
     if (lane == 31) {
@@ -726,6 +727,7 @@ __device__ __forceinline__ void tm_chain_column(SM& sm, const KParams<V>& p, int
         for (int e = 0; e < E; ++e) acc[e] = acc[e] + from_bits<V>(static_cast<uint32_t>(w[e]));
     }
     if (I == p.R - 1 && ch.rank + 1 < ch.nranks) {
+        SAT_JITTER_WARP();
         if (!bp_ok) {
             if (lane == 0)
                 sat_spin_until(static_cast<long long>(ld_relaxed_sys_u32(ch.peer_done[ch.rank] + ch.rank + 1)) >=
@@ -828,6 +830,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                                                                                     bp_ok);
             }
             if (!cin && __all_sync(kFull, pend == 0u)) {
+                SAT_JITTER_WARP();
                 // carries -> smem, raise the flag, then publish the inclusive words of the rows / columns
                 // whose local aggregates are already in
 #pragma unroll
@@ -856,6 +859,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                 progress = true;
             }
             if (!Cfg::CHAIN && ROW && cin && !ddone && !lpub) {  // Step 3.1: GLS, published as a local corner word
+                SAT_JITTER_WARP();
                 int go = 0;
                 if (lane == 31 && flag(&sm.cdone[s]) == k + 1 && flag(&sm.lw[s][NW - 1]) == k + 1) {
                     __threadfence_block();
@@ -873,6 +877,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
                 __nanosleep(32);
             }
         }
+        SAT_JITTER_WARP();
         // ---- Step 3.3 (GS, by whoever comes last) and the hand-off
         if (ROW && Cfg::CHAIN) {
             // corner = GS(I-1,J-1) = sum of X(I,J') over J' < J; then XG(I,J) = corner + X(I,J) = GS(I-1,J),
@@ -1070,6 +1075,10 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 const bool valid = t < p.ntiles;
                 TileInfo ti{t, 0, 0, 0};
                 if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
+                if (TMA && valid && p.l2_prefetch) {  // warm L2 while the tile waits for an input stage
+#pragma unroll
+                    for (int bx = 0; bx < Cfg::NB; ++bx) tma_prefetch_2d(&map_in, ti.J * TC + bx * Cfg::TB, ti.I * TR);
+                }
                 sm.info[ta.s] = ti;
                 if (!valid) {
                     *reinterpret_cast<volatile int*>(&sm.end_n) = ta.k;

@@ -75,7 +75,7 @@ def main() -> int:
                 note(f"variant {vi} carry row rep {rep}")
                 a = satgen.gen_host(700, 900, seed=77 + rep, dist="u32")
                 top = 300
-                carry = oracle.col_prefix_u32(a[:top])[-1].view(np.int32)
+                carry = oracle.sat_i32(a)[top - 1]  # the SAT row above the strip (sat()'s carry argument)
                 got = sat.sat(torch.from_numpy(np.ascontiguousarray(a[top:])).to(dev),
                               carry=torch.from_numpy(carry.copy()).to(dev)).cpu().numpy()
                 want = oracle.sat_i32(a)[top:]

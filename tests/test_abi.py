@@ -61,7 +61,8 @@ def test_variants_and_tuning(sat):
     with pytest.raises(sat.SatError):
         sat.set_tuning(n, 0, 0)
     with pytest.raises(sat.SatError):
-        sat.set_tuning(-1, 3, 0)
+        sat.set_tuning(-1, 4, 0)
+    sat.set_tuning(-1, 3 | (8 << 8), 0)  # anti-diagonal order of 8-tall tile groups (chained strips)
     with pytest.raises(sat.SatError):
         sat.set_tuning(-1, 0x201 | 0x10000, 0)
     sat.set_tuning(-1, 0x200, 0)  # anti-diagonal order of 2-tile groups
