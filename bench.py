@@ -557,7 +557,66 @@ def run_extras(args, sat, satgen, torch, x, peak) -> dict:
                                  "overhead_pct": (t_sat - t_cp) / t_cp * 100.0, "gbs": gbs, "frac": gbs / peak,
                                  "note": "in place; 5 launches between CUDA events"}
     out["chain_64k"] = chain_projection(torch, sat, satgen, n, t_sat)
+    out["next_paths_32k"] = next_paths(torch, sat, satgen, 32768, peak)
     return out
+
+
+def next_paths(torch, sat, satgen, n, peak) -> dict:
+    """SURVEY Sec. 8(f) rows beyond the hot path, device time at n x n (median of 10 after 3 warm-ups),
+    algorithmic GB/s against the measured copy peak and a same-bytes torch copy: u8 -> uint32 integral
+    image (NEXT-3, 1 + 4 B/elem; yardstick the u8 -> int32 widening copy), fp32 -> fp64 SAT and SAVSM
+    moments (NEXT-3, 4 + 8 B/elem; yardstick the fp32 -> fp64 widening copy), box filter r = 8 / 64
+    (NEXT-4, 4 + 4 B/elem), batched 256^2 int32 and u8 (NEXT-2)."""
+    import statistics
+
+    def med(fn, reps=10):
+        for _ in range(3):
+            fn()
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(reps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            fn()
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        return statistics.median(ts)
+
+    def entry(ms, bpe, yard_ms, yard):
+        gbs = n * n * bpe / (ms / 1e3) / 1e9
+        return {"ms": ms, "gbs": gbs, "frac": gbs / peak, "bytes_per_elem": bpe, "yardstick": yard,
+                "yardstick_ms": yard_ms, "vs_yardstick": ms / yard_ms}
+
+    res = {"n": n}
+    t = torch.empty((n, n), dtype=torch.int32, device="cuda")
+    out = torch.empty((n, n), dtype=torch.int32, device="cuda")
+    satgen.fill_tensor(t, 1451, "u8")
+    img = t.to(torch.uint8)
+    cp5 = med(lambda: out.copy_(img))
+    res["u8_integral_image"] = entry(med(lambda: sat.sat_u8(img, out=out)), 5, cp5, "u8 -> int32 copy_")
+    res["batched_u8_16384x256x256"] = entry(med(lambda: sat.sat_batched_u8(img.view(-1, 256, 256),
+                                                                            out=out.view(-1, 256, 256))),
+                                            5, cp5, "u8 -> int32 copy_")
+    del img
+    satgen.fill_tensor(t, 1447, "u32")
+    cp8 = med(lambda: out.copy_(t))
+    res["batched_i32_16384x256x256"] = entry(med(lambda: sat.sat_batched(t.view(-1, 256, 256),
+                                                                         out=out.view(-1, 256, 256))),
+                                             8, cp8, "int32 copy_")
+    res["box_sum_r8"] = entry(med(lambda: sat.box_sum(t, 8, 8, out=out)), 8, cp8, "int32 copy_")
+    res["box_sum_r64"] = entry(med(lambda: sat.box_sum(t, 64, 64, out=out)), 8, cp8, "int32 copy_")
+    del out
+    satgen.fill_tensor(t, 1447, "f01")
+    xf = t.view(torch.float32)
+    y64 = torch.empty((n, n), dtype=torch.float64, device="cuda")
+    cp12 = med(lambda: y64.copy_(xf))
+    res["f32_f64_sat"] = entry(med(lambda: sat.sat_f64(xf, out=y64)), 12, cp12, "fp32 -> fp64 copy_")
+    ym = y64.view(torch.float32).view(n, n, 2)
+    res["moments_f32"] = entry(med(lambda: sat.sat_moments(xf, out=ym)), 12, cp12, "fp32 -> fp64 copy_")
+    del t, xf, y64, ym
+    torch.cuda.empty_cache()
+    return res
 
 
 def chain_projection(torch, sat, satgen, n, single_ms) -> dict:

@@ -536,7 +536,11 @@ def test_sharded_nccl_single_rank():
                                                ((64, 1000), None, 40, 1), ((1009, 203), 208, 12, 12),
                                                ((50, 60), None, 100, 100), ((300, 516), None, 3, 5),
                                                ((40, 3001), 3004, 2, 700), ((33, 2500), None, 1, 1500),
-                                               ((20, 5000), None, 25, 0), ((7, 4), None, 0, 3)])
+                                               ((20, 5000), None, 25, 0), ((7, 4), None, 0, 3),
+                                               # band kernel: many panels / bands, halos across band tops
+                                               ((4096, 8192), None, 8, 8), ((2048, 8192), None, 64, 64),
+                                               ((3000, 33000), None, 2, 70), ((10000, 300), 304, 50, 3),
+                                               ((5000, 1200), None, 0, 0)])
 def test_box_sum_int32_bit_exact(sat, shape, pitch, rh, rw):
     b = satgen.gen_host(*shape, seed=31 + shape[0], dist="u32")  # any matrix is a valid operand of P:48
     buf, bd = dev_copy(b, pitch)
