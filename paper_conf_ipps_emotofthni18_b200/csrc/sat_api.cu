@@ -837,6 +837,59 @@ sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, in
     if (gy > 65535) gy = 65535;
     const dim3 grid(static_cast<unsigned>(gx), static_cast<unsigned>(gy));
     const bool vec = ((reinterpret_cast<uintptr_t>(out) & 15u) == 0) && ((pitch * 4) % 16 == 0);
+    // band kernel (production): one wave of sms x occ blocks cut into px column panels x bands row bands,
+    // the fewest bands (least re-read halo) whose panel is >= 128 columns wide and whose two rings of
+    // kBandQ x kBandRows row segments fit the shared memory of `occ` blocks per SM
+    if (vec && ((reinterpret_cast<uintptr_t>(b) & 15u) == 0) && cols % 4 == 0 && rows < (int64_t(1) << 31) - 1 &&
+        rh < (1 << 28) && rw < (1 << 20)) {
+        using CfgB = sat::BandCfg<8, 1>;  // 8 rows per slot, one slot ahead (measured: 4 blocks/SM, 32K^2 r = 8:
+                                          // 1.62 ms; <16, 1> at 2 blocks/SM 2.42 ms; <4, 4> 2.45 ms; <2, 4> 2.93 ms)
+        static const int band_occ_max = [] {
+            const char* e = std::getenv("SAT_BOX_BAND_OCC");  // tuning switch (0 = staged kernel)
+            return e ? std::atoi(e) : 8;
+        }();
+        // only at 4 blocks per SM (fewer leave the band walk latency-bound: r = 64 at 3 blocks/SM 2.87 ms vs
+        // 2.58 ms staged) and while the rows re-read as u stay in L2 (bands x (2 rh + 1) rows <= 48 MB)
+        for (int occ : {4}) {
+            if (occ > band_occ_max) continue;
+            const int64_t S = static_cast<int64_t>(sms) * occ;
+            const size_t limit = (228 * 1024) / occ - 1024;
+            for (int64_t bands = 1; bands <= S && bands <= rows; ++bands) {
+                if (S % bands) continue;
+                const int64_t px = S / bands;
+                const int64_t W = ((cols + px - 1) / px + 3) & ~int64_t(3);
+                if (W < 128 && px > 1) continue;
+                const int64_t segw = (W + 2 * rw + 8 + 3) & ~int64_t(3);  // 16-byte segment rows
+                const size_t bytes = CfgB::smem(segw);
+                if (bytes > limit) break;  // more bands only widen the panels
+                if (static_cast<double>(bands) * (2 * rh + 1) * cols * 4 > 48.0 * (1 << 20)) break;
+                const int64_t H = (rows + bands - 1) / bands;
+                const dim3 g(static_cast<unsigned>((cols + W - 1) / W), static_cast<unsigned>((rows + H - 1) / H));
+                auto go = [&](auto cfg) -> cudaError_t {
+                    using C = decltype(cfg);
+                    const void* k = dt == SAT_INT32 ? reinterpret_cast<const void*>(&sat::box_band_kernel<uint32_t, C>)
+                                                    : reinterpret_cast<const void*>(&sat::box_band_kernel<float, C>);
+                    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                         static_cast<int>(bytes));
+                    if (e != cudaSuccess) return e;
+                    if (dt == SAT_INT32)
+                        sat::box_band_kernel<uint32_t, C><<<g, 256, bytes, st>>>(
+                            static_cast<const uint32_t*>(b), static_cast<uint32_t*>(out), static_cast<int>(rows), cols,
+                            pitch, static_cast<int>(rh), static_cast<int>(rw), static_cast<int>(W), static_cast<int>(H),
+                            static_cast<int>(segw));
+                    else
+                        sat::box_band_kernel<float, C><<<g, 256, bytes, st>>>(
+                            static_cast<const float*>(b), static_cast<float*>(out), static_cast<int>(rows), cols, pitch,
+                            static_cast<int>(rh), static_cast<int>(rw), static_cast<int>(W), static_cast<int>(H),
+                            static_cast<int>(segw));
+                    return cudaGetLastError();
+                };
+                cudaError_t e = go(CfgB{});
+                if (e != cudaSuccess) return cuda_fail(e, "box_band_kernel");
+                return SAT_OK;
+            }
+        }
+    }
     // staged kernel: both pointers 16-byte aligned and kBoxBufs pairs of row segments in 48 KB
     const int64_t nv = (sat::kBoxPanel + 2 * rw + 8) / 4 + 1;
     const size_t smem = static_cast<size_t>(nv) * 4 * 4 * 2 * sat::kBoxBufs;

@@ -141,6 +141,127 @@ __global__ void __launch_bounds__(kBoxThreads) box_sum_smem_kernel(const V* __re
     asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
 
+// Band box filter (production): the matrix is cut into gridDim.x column panels of W output columns and
+// gridDim.y row bands of H output rows, one block each, sized by the host so the grid is one full wave
+// (blocks = SMs x resident blocks per SM).  A block walks its band top to bottom; output row i needs the
+// SAT row segments d = min(i + rh, rows - 1) and u = i - rh - 1 (columns [p0 - rw - 1, p0 + W - 1 + rw]).
+// Thread 0 fetches both with 1-D bulk copies (TMA engine, one instruction per segment, completion on the
+// ring slot's mbarrier), RB output rows per ring slot, AHEAD slots ahead; a thread evaluates its column
+// for the slot's RB rows as RB independent chains with hoisted offsets.  Measured at 32K^2 int32, r = 8
+// (tools/bench_box.py): row-at-a-time variants ran at 1.1-1.5 TB/s (instruction-issue
+// bound: ncu issue slots 68% busy at ~50 instructions per output); <8, 1> at 4 blocks per SM 1.62 ms =
+// 5.3 TB/s of the algorithmic 8 B/elem, with ncu DRAM read + write 1.02x algorithmic (the strided-row
+// staged kernel below reads the SAT twice from DRAM: 12.9 GB for 8.6 GB algorithmic).
+// Row d is new data (one DRAM read per SAT row and band); row u is the row d of 2 rh + 1 output rows
+// earlier -- an L2 hit while the concurrent bands' working set, bands x (2 rh + 1) rows x cols x 4 B, fits
+// in L2 (32K columns, rh = 64, two bands: 33 MB of 126 MB).  All blocks walk rows top-down at about the
+// same rate, so the panels' horizontal halos (2 rw + 1 columns, read by both neighbours) are L2 hits too.
+// Segment columns outside [0, cols) are zeroed once and never copied.  P:48 is evaluated left to right as
+// box_sum_kernel; columns < 0, rows < 0 read as 0.  Requires 16-byte aligned b, pitch % 4 == 0,
+// cols % 4 == 0 (whole 16-byte bulk-copy granules).
+// RB output rows per ring slot (one barrier and one mbarrier wait per slot), AHEAD slots in flight ahead of
+// the one being evaluated, Q = AHEAD + 2 ring slots (in flight, read now, read by laggards)
+template <int RB_, int AHEAD_>
+struct BandCfg {
+    static constexpr int RB = RB_, AHEAD = AHEAD_, Q = AHEAD_ + 2;
+    static constexpr size_t smem(int64_t segw) { return 256 + static_cast<size_t>(2) * Q * RB * segw * 4; }
+};
+
+template <typename V, typename Cfg>
+__global__ void __launch_bounds__(256) box_band_kernel(const V* __restrict__ b, V* __restrict__ out, int rows,
+                                                       int64_t cols, int64_t pitch, int rh, int rw, int W, int H,
+                                                       int segw) {
+    constexpr int Q = Cfg::Q, RB = Cfg::RB, kBandAhead = Cfg::AHEAD;
+    extern __shared__ __align__(128) unsigned char band_smem[];
+    uint64_t* full = reinterpret_cast<uint64_t*>(band_smem);  // [Q] mbarriers
+    V* ringD = reinterpret_cast<V*>(band_smem + 256);           // [Q][RB][segw]
+    V* ringU = ringD + Q * RB * segw;                           // [Q][RB][segw]
+    const int64_t p0 = static_cast<int64_t>(blockIdx.x) * W;
+    const int i0 = static_cast<int>(blockIdx.y) * H;
+    if (p0 >= cols || i0 >= rows) return;  // uniform per block
+    const int i1 = i0 + H < rows ? i0 + H : rows;
+    const int64_t pend = p0 + W < cols ? p0 + W : cols;
+    const int64_t a0 = (p0 - rw - 1) >= 0 ? ((p0 - rw - 1) & ~int64_t(3)) : -((-(p0 - rw - 1) + 3) & ~int64_t(3));
+    const int64_t hi = cols - 1;
+    const int64_t lo_c = a0 > 0 ? a0 : 0;                                  // first valid column of a segment
+    const int64_t hi_c = a0 + segw < cols ? a0 + segw : cols;              // one past the last valid column
+    const uint32_t seg_bytes = static_cast<uint32_t>((hi_c - lo_c) * sizeof(V));
+    const int seg_off = static_cast<int>(lo_c - a0);
+    // zero both rings (the invalid columns stay zero: copies only ever write [lo_c, hi_c)), init barriers
+    for (int k = threadIdx.x; k < 2 * Q * RB * segw; k += blockDim.x) ringD[k] = V(0);
+    if (threadIdx.x == 0) {
+        for (int q = 0; q < Q; ++q) mbar_init(&full[q], 1);
+        fence_mbar_init();
+    }
+    fence_proxy_async_smem();  // the zeros (generic proxy) before the bulk copies (async proxy)
+    __syncthreads();
+    const int nslots = (i1 - i0 + RB - 1) / RB;
+    auto issue_slot = [&](int n, int slot) {  // thread 0: segments of output rows i0 + n*RB .. + RB - 1
+        if (n >= nslots) return;
+        const int ia = i0 + n * RB, ib = ia + RB < i1 ? ia + RB : i1;
+        uint32_t bytes = 0;
+        for (int i = ia; i < ib; ++i) bytes += (i - rh - 1 >= 0) ? 2 * seg_bytes : seg_bytes;
+        mbar_arrive_expect_tx(&full[slot], bytes);
+        for (int i = ia; i < ib; ++i) {
+            const int d = i + rh < rows - 1 ? i + rh : rows - 1, u = i - rh - 1;
+            V* sd = ringD + (slot * RB + (i - ia)) * segw + seg_off;
+            bulk_load_1d(sd, b + static_cast<int64_t>(d) * pitch + lo_c, seg_bytes, &full[slot]);
+            if (u >= 0)
+                bulk_load_1d(ringU + (slot * RB + (i - ia)) * segw + seg_off, b + static_cast<int64_t>(u) * pitch + lo_c,
+                             seg_bytes, &full[slot]);
+        }
+    };
+    if (threadIdx.x == 0)
+        for (int n = 0; n < kBandAhead; ++n) issue_slot(n, n);
+    const int64_t jcol = p0 + threadIdx.x;  // the fast path's column of this thread
+    const int kr0 = static_cast<int>((jcol + rw < hi ? jcol + rw : hi) - a0), kl0 = static_cast<int>(jcol - rw - 1 - a0);
+    int slot = 0;
+    uint32_t phase = 0;
+    for (int n = 0; n < nslots; ++n) {
+        if (threadIdx.x == 0) {  // that slot was last read for slot number n + kBandAhead - Q = n - 2 (barrier below)
+            const int f = slot + kBandAhead < Q ? slot + kBandAhead : slot + kBandAhead - Q;
+            issue_slot(n + kBandAhead, f);
+        }
+        mbar_wait(&full[slot], phase);
+        const int ia = i0 + n * RB, ib = ia + RB < i1 ? ia + RB : i1;
+        const V* D = ringD + slot * RB * segw;
+        const V* U = ringU + slot * RB * segw;
+        if (ib - ia == RB && ia - rh - 1 >= 0 && W <= static_cast<int>(blockDim.x)) {
+            // fast path (every slot but the band's first and last few): one column per thread, all RB rows
+            // present and below the top halo -- RB independent load / add / store chains, offsets hoisted
+            if (jcol < pend) {
+                V* dst = out + static_cast<int64_t>(ia) * pitch + jcol;
+#pragma unroll
+                for (int rr = 0; rr < RB; ++rr) {
+                    const V dr = D[rr * segw + kr0], dl = D[rr * segw + kl0];
+                    const V ur = U[rr * segw + kr0], ul = U[rr * segw + kl0];
+                    __stcs(dst + rr * pitch, ((dr - ur) - dl) + ul);
+                }
+            }
+        } else {
+            for (int64_t j = p0 + threadIdx.x; j < pend; j += blockDim.x) {
+                const int64_t r = j + rw < hi ? j + rw : hi;
+                const int kr = static_cast<int>(r - a0), kl = static_cast<int>(j - rw - 1 - a0);
+                V* dst = out + static_cast<int64_t>(ia) * pitch + j;
+#pragma unroll
+                for (int rr = 0; rr < RB; ++rr) {
+                    if (ia + rr < ib) {
+                        const V dr = D[rr * segw + kr], dl = D[rr * segw + kl];
+                        const bool has_u = ia + rr - rh - 1 >= 0;
+                        const V ur = has_u ? U[rr * segw + kr] : V(0), ul = has_u ? U[rr * segw + kl] : V(0);
+                        __stcs(dst + rr * pitch, ((dr - ur) - dl) + ul);
+                    }
+                }
+            }
+        }
+        if (++slot == Q) {
+            slot = 0;
+            phase ^= 1u;
+        }
+        __syncthreads();  // every thread is done with this slot before it is refilled (two slots later)
+    }
+}
+
 // Batched rectangle queries: rects[k] = (u, d, l, r) in the convention of P:48 (u < i <= d,
 // l < j <= r).  Indices are clamped into [-1, rows-1] / [-1, cols-1] (memory safety); an empty
 // rectangle (u >= d or l >= r after clamping) gives 0.
