@@ -105,9 +105,9 @@ struct Family<sat::WsCfg<TR, NW, ST, NT, NQ, FLAGS>> {
 #endif
 
 template <int NW, int IN, int NQ, int NT, int WPUB, int D, int DIRECT, int QS, int TR, int TC, int LB, int CT, int DW,
-          int CH>
-struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT, DW, CH>> {
-    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT, DW, CH>;
+          int CH, int MINB, int RW2>
+struct Family<sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT, DW, CH, MINB, RW2>> {
+    using Cfg = sat::TmCfg<NW, IN, NQ, NT, WPUB, D, DIRECT, QS, TR, TC, LB, CT, DW, CH, MINB, RW2>;
     static constexpr int box_cols = Cfg::TB;
     static constexpr int out_box_rows = Cfg::OBR;
     static constexpr int threads = Cfg::THREADS;
@@ -234,19 +234,27 @@ enum : int { kVarClassic = 0, kVarTm128 = 1, kVarU8 = 2, kVarFlat = 3, kVarChain
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),                   // 0: classic, 64 x 128 tiles (small matrices)
-        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>, true>(),            // 1: TMEM-parked, 128 x 128 tiles
+        // 1: TMEM-parked, 128 x 128 tiles, two row walker warps (even / odd tiles): 4K^2 38.3 -> 34.8 us,
+        //    8K^2 103.5 -> 99.5 us (the row + diagonal walks are the medium sizes' long pole)
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 2, 0, 4, 0, 1, 1>, true>(),
         make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>, true>(),            // 2: u8 integral images (4 stages of 16 KiB)
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 3: TMEM-parked, flat 64 x 256 tiles
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32, 1>>(),  // 4: chained strips (sat_compute_chained only)
-        // round-2 candidates (medium sizes): 8 compute warps on 128 x 128 tiles, wider look-back windows
+#if SAT_EXPERIMENTAL
+        // tuning builds only (numbering continues after the shipped variants 0-4):
+        // round-2 candidates, measured and not shipped (medium sizes): 8 compute warps on 128 x 128 tiles, wider look-back windows
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 2>>(),            // 5
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 4, 0, 32>>(),     // 6
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32>>(),     // 7
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 4>>(),      // 8
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 0, 32>>(),      // 9: flat, diagonal 32
         make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),                // 10: flat, tile ring of 8
-#if SAT_EXPERIMENTAL
-        make_variant<sat::TmCfg<16, 2, 5>>(),  // 5: walkers publish (blocking ws_walker)
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>, true>(),             // round-1 variant 1 (one row walker)
+        make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 0, 4, 0, 1, 1>>(),  // flat + two row walkers
+        // round-2 medium-size candidates: 64 x 128 tiles (32 KiB), 2 CTAs per SM (registers capped at 85)
+        make_variant<sat::TmCfg<8, 2, 5, 1, 3, 4, 0, 0, 64, 128, 2, 0, 4, 0, 2>>(),    // 11
+        make_variant<sat::TmCfg<8, 2, 5, 1, 3, 4, 0, 0, 64, 128, 4, 0, 32, 0, 2>>(),   // 12
+        make_variant<sat::TmCfg<16, 2, 5>>(),  // walkers publish (blocking ws_walker)
         make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch | sat::kWsDefer | sat::kWsDirect>>(),  // 6
         make_variant<sat::WsCfg<128, 16, 3, 1, 5, sat::kWsPrefetch>>(),  // 7: warp-specialised, TMA store
         make_variant<sat::TmCfg<16, 2, 5, 1, 2>>(),  // 8
@@ -283,10 +291,11 @@ int g_max_ctas = 0;
 int auto_variant(int64_t rows, int64_t cols) {
     // measured device times (tools/graph_sweep.py, tools/sweep_variants.py): up to
     // ~1.4K x 1.4K (<= 128 tiles of 128^2) the classic kernel with 64 x 128 tiles has the shortest
-    // latency; above, the TMEM-parked kernel with decoupled walkers (parking depth 4) on flat
-    // 64 x 256 tiles
+    // latency; up to 8K x 8K the TMEM-parked kernel on 128 x 128 tiles with two row walkers (round 2:
+    // 4K^2 34.8 us, 8K^2 99.5 us vs 37.4 / 102.1 on flat tiles); above, the TMEM-parked kernel with
+    // decoupled walkers (parking depth 4) on flat 64 x 256 tiles
     const int64_t n = rows * cols;
-    return n <= (int64_t(1) << 21) ? kVarClassic : (n <= (int64_t(1) << 25) ? kVarTm128 : kVarFlat);
+    return n <= (int64_t(1) << 21) ? kVarClassic : (n <= (int64_t(1) << 26) ? kVarTm128 : kVarFlat);
 }
 
 // L2 prefetch of a tile's boxes when the loader acquires it (cp.async.bulk.prefetch.tensor): the DRAM read

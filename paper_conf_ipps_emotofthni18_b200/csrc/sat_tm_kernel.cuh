@@ -32,8 +32,10 @@ namespace sat {
 // TR_ x TC_ tiles: TC_ = 128 * G (a lane owns G chunks of 4 columns, 128 apart); flat tiles (TC_ > 128)
 // keep the tile's 64 KiB but make every DRAM row visit 4 B * TC_ long (tile shape).
 template <int NW_, int IN_, int NQ_, int NT_ = 1, int WPUB_ = 1, int D_ = 2, int DIRECT_ = 0, int QS_ = 0,
-          int TR_ = 128, int TC_ = 128, int LB_ = 2, int CT_ = 0, int DW_ = 4, int CH_ = 0>
+          int TR_ = 128, int TC_ = 128, int LB_ = 2, int CT_ = 0, int DW_ = 4, int CH_ = 0, int MINB_ = 1, int RW2_ = 0>
 struct TmCfg {
+    static constexpr int MINB = MINB_;              // resident CTAs per SM the registers are capped for
+    static constexpr int RW2 = RW2_;                // 1: two row walker warps, even / odd tiles
     // Chained strip partition (sat_compute_chained): column-major tile order, column carries = strip-local
     // vertical look-back + the upstream ranks' strip column sums from the inbox, corners by a horizontal
     // look-back; bottom tiles push their strip column sums to the downstream ranks.
@@ -63,11 +65,12 @@ struct TmCfg {
     static constexpr int TM_COLS_PER_SLOT = (NW / 4) * NREG;
     static constexpr int TM_COLS = D * TM_COLS_PER_SLOT <= 32 ? 32 : D * TM_COLS_PER_SLOT <= 64 ? 64
                                  : D * TM_COLS_PER_SLOT <= 128 ? 128 : D * TM_COLS_PER_SLOT <= 256 ? 256 : 512;
-    static constexpr int ROW_WARP = NW, COL_WARP = NW + 1, STORE_WARP = NW + 2, LOAD_WARP = NW + 3;
-    static constexpr int THREADS = (NW + 4) * 32;
+    static constexpr int ROW_WARP = NW, COL_WARP = NW + 1, STORE_WARP = NW + 2, LOAD_WARP = NW + 3, ROW2_WARP = NW + 4;
+    static constexpr int THREADS = (NW + 4 + RW2) * 32;
     static_assert(NW % 4 == 0 && TR % NW == 0 && RPW % 4 == 0, "compute warps cover the 4 TMEM lane quarters");
     static_assert(NREG == 16 || NREG == 32 || NREG == 64, "tcgen05 32x32b.x16 / .x32 parking");
-    static_assert(TC % 128 == 0 && TC % TB == 0 && TR >= 32 && TR * TC == 128 * 128, "64 KiB tiles, TC = 128 G");
+    static_assert(TC % 128 == 0 && TC % TB == 0 && TR >= 32 && (TR * TC == 128 * 128 || (TR * TC == 64 * 128 && MINB == 2)),
+                  "64 KiB tiles (32 KiB tiles for 2 CTAs per SM), TC = 128 G");
     static_assert(!SBAND || !QS, "flat tiles: whole-tile TMA stores");
     static_assert(!CT || (TC == 256 && !DIRECT), "contiguous lane columns: 64 x 256 tiles");
     static_assert(D >= 2 && D * TM_COLS_PER_SLOT <= 512, "TMEM columns");
@@ -762,7 +765,8 @@ __device__ __forceinline__ void tm_chain_column(SM& sm, const KParams<V>& p, int
 // the first GS word (reading R8) instead of waiting for GS(I-1,J-1): no chain in any of the
 // three directions waits for a neighbour's completion.
 template <typename V, typename Cfg, bool ROW, typename TIn>
-__device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, uint32_t epoch, int lane) {
+__device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, uint32_t epoch, int lane,
+                                          int first = 0, int stride = 1) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, RPW = Cfg::RPW, NW = Cfg::NW;
     constexpr int E = ROW ? Cfg::ER : Cfg::EC;
     constexpr int DW = Cfg::DW;  // diagonal predecessors polled per round
@@ -771,7 +775,9 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
     const uint64_t pol = policy_evict_last();
     auto flag = [&](const int* f) { return *reinterpret_cast<const volatile int*>(f); };
     bool bp_ok = false;  // chain mode: the downstream ranks have released this call's inbox half
-    for (Slot<Cfg::NQ> nx;; nx.next()) {
+    Slot<Cfg::NQ> nx;
+    for (int f = 0; f < first; ++f) nx.next();
+    for (;; [&] { for (int f = 0; f < stride; ++f) nx.next(); }()) {
         if (!wait_acquired(sm, nx.s, nx.ph, nx.k)) break;
         const TileInfo ti = sm.info[nx.s];
         if (ti.t >= p.ntiles) break;
@@ -918,7 +924,7 @@ __device__ __forceinline__ void tm_walker(TmSmem<V, Cfg, TIn>& sm, const KParams
 }
 
 template <typename V, typename Cfg, bool TMA, bool CARRY, typename TIn = V>
-__global__ void __launch_bounds__(Cfg::THREADS, 1)
+__global__ void __launch_bounds__(Cfg::THREADS, Cfg::MINB)
 sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant__ CUtensorMap map_out,
               const KParams<V> p) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, IN = Cfg::IN;
@@ -997,7 +1003,9 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
         if constexpr (!Cfg::DECOUPLED) ws_walker<V, Cfg, true>(sm, p, epoch, lane);
         else
 #endif
-        tm_walker<V, Cfg, true, TIn>(sm, p, epoch, lane);
+        tm_walker<V, Cfg, true, TIn>(sm, p, epoch, lane, 0, Cfg::RW2 ? 2 : 1);
+    } else if (Cfg::RW2 && warp == Cfg::ROW2_WARP) {
+        tm_walker<V, Cfg, true, TIn>(sm, p, epoch, lane, 1, 2);  // the odd tiles' row / diagonal walks
     } else if (warp == Cfg::COL_WARP) {
 #if SAT_EXPERIMENTAL
         if constexpr (!Cfg::DECOUPLED) ws_walker<V, Cfg, false>(sm, p, epoch, lane);
