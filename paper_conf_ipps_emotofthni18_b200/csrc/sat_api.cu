@@ -250,6 +250,9 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 0, 32>>(),      // 9: flat, diagonal 32
         make_variant<sat::TmCfg<8, 2, 8, 1, 3, 4, 0, 0, 64, 256>>(),                // 10: flat, tile ring of 8
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4>, true>(),             // round-1 variant 1 (one row walker)
+        make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4, 0, 0, 128, 128, 2, 0, 4, 0, 1, 1>, true>(),  // u8 + two row walkers
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32, 1, 1, 1>>(),       // chain, 16 warps + RW2
+        make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32, 1>>(),             // chain, 16 warps
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256, 2, 0, 4, 0, 1, 1>>(),  // flat + two row walkers
         // round-2 medium-size candidates: 64 x 128 tiles (32 KiB), 2 CTAs per SM (registers capped at 85)
         make_variant<sat::TmCfg<8, 2, 5, 1, 3, 4, 0, 0, 64, 128, 2, 0, 4, 0, 2>>(),    // 11
@@ -855,11 +858,15 @@ sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, in
                                           // 1.62 ms; <16, 1> at 2 blocks/SM 2.42 ms; <4, 4> 2.45 ms; <2, 4> 2.93 ms)
         static const int band_occ_max = [] {
             const char* e = std::getenv("SAT_BOX_BAND_OCC");  // tuning switch (0 = staged kernel)
-            return e ? std::atoi(e) : 8;
+            return e ? std::atoi(e) : 4;
         }();
         // only at 4 blocks per SM (fewer leave the band walk latency-bound: r = 64 at 3 blocks/SM 2.87 ms vs
         // 2.58 ms staged) and while the rows re-read as u stay in L2 (bands x (2 rh + 1) rows <= 48 MB)
-        for (int occ : {4}) {
+        static const int band_cfg = [] {  // tuning switch: 0 = <8,1> (default), 1 = <6,2>, 2 = <4,3>
+            const char* e = std::getenv("SAT_BOX_BAND_CFG");
+            return e ? std::atoi(e) : 0;
+        }();
+        for (int occ : {band_occ_max >= 5 ? 5 : 4}) {
             if (occ > band_occ_max) continue;
             const int64_t S = static_cast<int64_t>(sms) * occ;
             const size_t limit = (228 * 1024) / occ - 1024;
@@ -869,7 +876,8 @@ sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, in
                 const int64_t W = ((cols + px - 1) / px + 3) & ~int64_t(3);
                 if (W < 128 && px > 1) continue;
                 const int64_t segw = (W + 2 * rw + 8 + 3) & ~int64_t(3);  // 16-byte segment rows
-                const size_t bytes = CfgB::smem(segw);
+                const size_t bytes = band_cfg == 1 ? sat::BandCfg<6, 2>::smem(segw)
+                                     : band_cfg == 2 ? sat::BandCfg<4, 3>::smem(segw) : CfgB::smem(segw);
                 if (bytes > limit) break;  // more bands only widen the panels
                 if (static_cast<double>(bands) * (2 * rh + 1) * cols * 4 > 48.0 * (1 << 20)) break;
                 const int64_t H = (rows + bands - 1) / bands;
@@ -893,7 +901,8 @@ sat_status_t box_impl(sat_dtype_t dt, const void* b, void* out, int64_t rows, in
                             static_cast<int>(segw));
                     return cudaGetLastError();
                 };
-                cudaError_t e = go(CfgB{});
+                cudaError_t e = band_cfg == 1 ? go(sat::BandCfg<6, 2>{}) : band_cfg == 2 ? go(sat::BandCfg<4, 3>{})
+                                                                       : go(CfgB{});
                 if (e != cudaSuccess) return cuda_fail(e, "box_band_kernel");
                 return SAT_OK;
             }
@@ -1059,7 +1068,7 @@ sat_status_t batched_impl(sat_dtype_t dt, const void* src, void* dst, int64_t ba
 // One staging buffer, copy-stream pair and event set per device.  `mu` is held for a whole
 // sat_compute_host call (through its final synchronisations), so concurrent calls on one device
 // run one after the other instead of sharing the buffer.
-constexpr int kHostMaxStrips = 16;
+constexpr int kHostMaxStrips = 64;
 struct Staging {
     std::mutex mu;
     void* buf = nullptr;
