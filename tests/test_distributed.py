@@ -1,8 +1,10 @@
 """Multi-process host logic of the strip-partitioned path (BASELINE.json configs[4]) on CPU with the
 gloo backend, world size 2 and 3: the NCCL id bootstrap, the strip partition check, and the carry
 exchange protocol (which ranks' column sums enter a rank's carry, in which order) replayed with the
-oracle's arithmetic through real torch.distributed collectives.  The device kernels of the same
-path are covered by tests/test_gpu_parity.py (fake exchange on one GPU, and a 1-rank NCCL run)."""
+oracle's arithmetic through real torch.distributed collectives.  On a GPU box,
+test_gather_path_multiprocess_libsat_kernels runs the same exchange with libsat's own device kernels in
+2 / 3 processes (gloo in place of ncclAllGather); the chained path's two-process CUDA IPC test is in
+tests/test_gpu_chain.py."""
 import os
 import socket
 import traceback
@@ -161,3 +163,39 @@ def test_chain_handle_exchange_gloo_world2():
         p.join(timeout=30)
     want = [bytes((r * 37 + i) % 256 for i in range(64)) for r in range(2)]
     assert out[0] == want and out[1] == want
+
+
+# ----------------------------------------------------------------------------- gather path through libsat's kernels
+def _w_gather_path_libsat(rank, world, rows, cols, seed, dist_name):
+    """The exchange of sat_compute_sharded with libsat's OWN device kernels in every process -- strip column
+    sums (sat_strip_colsum), carry row (sat_carry_prefix), single pass with the carry (sat_compute) --
+    and gloo standing in for ncclAllGather (this pool gives one GPU per call; NCCL refuses two ranks on one
+    device).  Each rank checks its strip against the oracle SAT of the whole matrix."""
+    import oracle
+    import paper_conf_ipps_emotofthni18_b200 as sat
+    import satgen
+
+    torch.cuda.set_device(0)
+    row0, n = sat.strip_bounds(rows, world, rank)
+    strip = satgen.gen_host(n, cols, seed, dist_name, row0=row0)
+    x = torch.from_numpy(strip).cuda()
+    colsum = sat.strip_colsum(x)
+    gathered = [torch.zeros(cols, dtype=x.dtype) for _ in range(world)]
+    dist.all_gather(gathered, colsum.cpu())
+    carry = sat.carry_prefix(torch.stack(gathered).cuda(), rank)
+    got = sat.sat(x, carry=carry).cpu().numpy()
+    full = satgen.gen_host(rows, cols, seed, dist_name)
+    if dist_name == "u32":
+        assert (got == oracle.sat_i32(full)[row0:row0 + n]).all()
+    else:
+        b, ab = oracle.sat_f32(full)
+        tol = oracle.f32_tolerance(ab, rows, cols)[row0:row0 + n]
+        assert (np.abs(got.astype(np.float64) - b[row0:row0 + n]) <= tol).all()
+    return n
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world,dist_name", [(2, "u32"), (3, "u32"), (2, "fsym")])
+def test_gather_path_multiprocess_libsat_kernels(world, dist_name):
+    res = _run(world, _w_gather_path_libsat, 2500, 3100, 4141 + world, dist_name)
+    assert sum(res.values()) == 2500
