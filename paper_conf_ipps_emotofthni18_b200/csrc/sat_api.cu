@@ -217,7 +217,7 @@ Variant make_variant() {
     v.prepare[SAT_FLOAT32] = &prepare_variant<float, Cfg>;
     if constexpr (HasBox<Family<Cfg>>::value) v.TB = Family<Cfg>::box_cols;
     else v.TB = Cfg::TC;
-    if constexpr (U8 && HasU8<Family<Cfg>>::value && Cfg::TC == 128 && !IsChain<Cfg>::value) {
+    if constexpr (U8 && HasU8<Family<Cfg>>::value && Cfg::TC <= 256 && !IsChain<Cfg>::value) {
         v.launch[kU8] = &launch_variant_u8<Cfg>;
         v.prepare[kU8] = &prepare_variant_u8<Cfg>;
     } else {
@@ -230,7 +230,7 @@ Variant make_variant() {
 // Shipped kernel variants (auto_variant picks among them; sat_set_tuning can force one, test hook).
 // Tuning builds (-DSAT_EXPERIMENTAL=1) append the configurations measured and not kept in round 1
 // (DESIGN.md Sec. 5), so that they can still be re-measured.
-enum : int { kVarClassic = 0, kVarTm128 = 1, kVarU8 = 2, kVarFlat = 3, kVarChain = 4 };
+enum : int { kVarClassic = 0, kVarTm128 = 1, kVarU8 = 2, kVarFlat = 3, kVarChain = 4, kVarU8Flat = 5 };
 const std::vector<Variant>& variants() {
     static const std::vector<Variant> vs = {
         make_variant<sat::TileCfg<64, 128, 8, 2>>(),                   // 0: classic, 64 x 128 tiles (small matrices)
@@ -240,8 +240,12 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>, true>(),            // 2: u8 integral images (4 stages of 16 KiB)
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 3: TMEM-parked, flat 64 x 256 tiles
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32, 1>>(),  // 4: chained strips (sat_compute_chained only)
+        // 5: u8 integral images on flat 64 x 256 tiles (4 stages of 16 KiB, 8 compute warps), above 2^25 pixels:
+        //    32K^2 1.145 -> 1.044 ms, 16K^2 0.331 -> 0.304 ms (tools/u8_probe.py; 3 / 6 stages, a ring of 8
+        //    and the 2-tile-group order measured no better)
+        make_variant<sat::TmCfg<8, 4, 7, 1, 3, 4, 0, 0, 64, 256>, true>(),
 #if SAT_EXPERIMENTAL
-        // tuning builds only (numbering continues after the shipped variants 0-4):
+        // tuning builds only (numbering continues after the shipped variants 0-5):
         // round-2 candidates, measured and not shipped (medium sizes): 8 compute warps on 128 x 128 tiles, wider look-back windows
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 2>>(),            // 5
         make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 4, 0, 32>>(),     // 6
@@ -565,7 +569,8 @@ sat_status_t make_plan(int64_t rows, int64_t cols, int64_t pitch, const void* sr
     } else {
         std::lock_guard<std::mutex> lk(g_mu);
         const bool forced = g_variant >= 0 && !variants()[g_variant].chain;  // chain configs: chained calls only
-        vi = forced ? g_variant : (u8 ? kVarU8 : auto_variant(rows, cols));
+        vi = forced ? g_variant
+                    : (u8 ? (rows * cols <= (int64_t(1) << 25) ? kVarU8 : kVarU8Flat) : auto_variant(rows, cols));
         order = (!forced && g_order == 0) ? auto_order(vi, cols) : g_order;
     }
     const Variant& v = variants()[vi];

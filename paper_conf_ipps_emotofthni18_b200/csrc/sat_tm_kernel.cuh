@@ -221,7 +221,6 @@ template <typename V, typename Cfg, bool TMA, typename TIn>
 __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<V>& p, const Slot<Cfg::IN>& sl,
                                          const Slot<Cfg::NQ>& tq, uint32_t epoch, int warp, int lane) {
     constexpr int TR = Cfg::TR, TC = Cfg::TC, NW = Cfg::NW, RPW = Cfg::RPW, G = Cfg::G, X = 4 * Cfg::G;
-    static_assert(sizeof(TIn) != 1 || TC == 128, "u8 tiles: 128 columns");
     const int s = sl.s;
     const int row0 = warp * RPW, col0 = lane * 4;  // this lane's columns: tm_cb<Cfg>(lane, g) + c
     SAT_CLK(c0);
@@ -238,14 +237,17 @@ __device__ __forceinline__ bool tm_local(TmSmem<V, Cfg, TIn>& sm, const KParams<
     const int par = tq.k & 1;
     V v[RPW][X];
     if constexpr (TMA && sizeof(TIn) == 1) {
-        // u8 pixels (integral image): a lane's 4 columns are one 32-bit word of the stage row
+        // u8 pixels (integral image): each of a lane's chunks of 4 columns is one 32-bit word of the stage row
+        static_assert(TC <= 256, "u8 tiles: one TMA box per row");
         const TIn* tile = sm.stage[s];
 #pragma unroll
-        for (int r = 0; r < RPW; ++r) {
-            const uint32_t w = *reinterpret_cast<const uint32_t*>(&tile[(row0 + r) * TC + col0]);
+        for (int r = 0; r < RPW; ++r)
 #pragma unroll
-            for (int c = 0; c < 4; ++c) v[r][c] = V((w >> (8 * c)) & 0xffu);
-        }
+            for (int g = 0; g < G; ++g) {
+                const uint32_t w = *reinterpret_cast<const uint32_t*>(&tile[(row0 + r) * TC + tm_cb<Cfg>(lane, g)]);
+#pragma unroll
+                for (int c = 0; c < 4; ++c) v[r][4 * g + c] = V((w >> (8 * c)) & 0xffu);
+            }
     } else if constexpr (TMA && Cfg::CT) {
         // two 16-byte halves per row, the lanes of each quarter-warp in swapped order (conflict-free)
         const TIn* tile = sm.stage[s];

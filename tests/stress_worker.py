@@ -83,13 +83,16 @@ def main() -> int:
                     raise AssertionError(f"variant {vi} carry row rep {rep}")
                 n += 1
             sat.set_tuning(-1, 0, 0)
-            # u8 integral images (variant 2)
-            for rows, cols in shapes[:2]:
-                img = satgen.gen_host(rows, cols, seed=50 + rep, dist="u8").astype(np.uint8)
-                note(f"u8 {rows}x{cols} rep {rep}")
-                got = sat.sat_u8(torch.from_numpy(img).to(dev)).cpu().numpy()
-                check(got, img, "u8", f"u8 {rows}x{cols} rep {rep}")
-                n += 1
+            # u8 integral images: 128 x 128 (variant 2) and flat 64 x 256 (variant 5) kernels
+            for uv in (2, 5):
+                sat.set_tuning(uv, 0, 0)
+                for rows, cols in shapes[:2]:
+                    img = satgen.gen_host(rows, cols, seed=50 + rep, dist="u8").astype(np.uint8)
+                    note(f"u8 variant {uv} {rows}x{cols} rep {rep}")
+                    got = sat.sat_u8(torch.from_numpy(img).to(dev)).cpu().numpy()
+                    check(got, img, "u8", f"u8 variant {uv} {rows}x{cols} rep {rep}")
+                    n += 1
+            sat.set_tuning(-1, 0, 0)
             # chained strips: 3 ranks, concurrent on their own streams (inbox pushes, polls, back-pressure)
             rows, cols, nr = 1500, 1300, 3
             note(f"chained strips rep {rep}")

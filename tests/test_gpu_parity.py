@@ -611,9 +611,12 @@ def test_query_errors(sat):
 # ----------------------------------------------------------------------------- u8 integral images (NEXT-3)
 @pytest.mark.parametrize("shape,spitch,opitch", [((1, 1), None, None), ((300, 517), None, None),
                                                  ((256, 256), 272, 260), ((1000, 2048), None, None),
-                                                 ((129, 131), 133, None), ((4096, 4096), None, None)])
-def test_u8_integral_image_bit_exact(sat, shape, spitch, opitch):
+                                                 ((129, 131), 133, None), ((4096, 4096), None, None),
+                                                 ((6000, 6000), None, None), ((777, 3001), 3008, 3004)])
+@pytest.mark.parametrize("variant", [-1, 5])  # auto; the flat-tile u8 kernel forced on every shape
+def test_u8_integral_image_bit_exact(sat, shape, spitch, opitch, variant):
     rows, cols = shape
+    sat.set_tuning(variant, 0, 0)
     a = satgen.gen_host(rows, cols, seed=rows * 7 + cols, dist="u8").astype(np.uint8)
     sp = cols if spitch is None else spitch
     op = cols if opitch is None else opitch
@@ -622,8 +625,11 @@ def test_u8_integral_image_bit_exact(sat, shape, spitch, opitch):
     src.copy_(torch.from_numpy(a).cuda())
     obuf = torch.full((rows * op + 64,), 0x5A5A5A5A, dtype=torch.int32, device="cuda")
     out = obuf[: rows * op].view(rows, op)[:, :cols]
-    sat.sat_u8(src, out=out)
-    torch.cuda.synchronize()
+    try:
+        sat.sat_u8(src, out=out)
+        torch.cuda.synchronize()
+    finally:
+        sat.set_tuning(-1, 0, 0)
     got = out.cpu().numpy().view(np.uint32)
     want = oracle.sat_u32(a.astype(np.uint32))
     assert (got == want).all()
