@@ -239,7 +239,9 @@ const std::vector<Variant>& variants() {
         make_variant<sat::TmCfg<16, 2, 7, 1, 3, 4, 0, 0, 128, 128, 2, 0, 4, 0, 1, 1>, true>(),
         make_variant<sat::TmCfg<16, 4, 9, 1, 3, 4>, true>(),            // 2: u8 integral images (4 stages of 16 KiB)
         make_variant<sat::TmCfg<8, 2, 6, 1, 3, 4, 0, 0, 64, 256>>(),    // 3: TMEM-parked, flat 64 x 256 tiles
-        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 8, 0, 32, 1>>(),  // 4: chained strips (sat_compute_chained only)
+        // 4: chained strips (sat_compute_chained only); look-back window 2 (64K^2 / 8 per rank: 0.739 ms; windows
+        //    of 4 / 8 0.740 / 0.756, diagonal window 4 0.783, a ring of 8 0.783, two row walkers 0.863)
+        make_variant<sat::TmCfg<8, 2, 7, 1, 3, 4, 0, 0, 128, 128, 2, 0, 32, 1>>(),
         // 5: u8 integral images on flat 64 x 256 tiles (4 stages of 16 KiB, 8 compute warps), above 2^25 pixels:
         //    32K^2 1.145 -> 1.044 ms, 16K^2 0.331 -> 0.304 ms (tools/u8_probe.py; 3 / 6 stages, a ring of 8
         //    and the 2-tile-group order measured no better)
@@ -1474,8 +1476,9 @@ SAT_API sat_status_t sat_chain_destroy(sat_chain_t chain) {
 // Tile order of a chained strip with R tile rows: anti-diagonal over groups of g vertically adjacent tiles
 // (order 3, tile_of_serial), g the largest of 8, 4, 2 dividing R: the strip's bottom tile of column J
 // resolves R/g group diagonals after its top tile -- the chain's lag per rank, (R/g) / (R/g + C) of a
-// strip -- and a column look-back (8 predecessors per poll round) spans the g - 1 tiles above in the group
-// plus the inclusive word of the group above.  SAT_CHAIN_ORDER overrides it (tuning: 2 = column-major).
+// strip -- and a column look-back spans the g - 1 tiles above in the group
+// plus the inclusive word of the group above (a few poll rounds).  SAT_CHAIN_ORDER overrides it (tuning:
+// 2 = column-major).
 int chain_order(int R) {
     if (const char* e = std::getenv("SAT_CHAIN_ORDER")) return std::atoi(e);
     for (int g : {8, 4, 2})
