@@ -4,6 +4,8 @@
   carry row, through the strip-partition pipeline with the NCCL all-gather replaced by a local stack,
   every row against the streaming oracle fed with the rows above;
 * the 64K x 64K single pass (configs[4] on one GPU), streamed row by row against the oracle;
+* the 64K x 64K chained strip partition over 8 emulated ranks (configs[4] as bench.py projects it), every
+  element;
 * 32K x 32K fp32 with the cancellation distribution U[-1,1) (configs[3]);
 * the aggregate words the kernels publish (Steps 2.A/2.B/3) against oracle.table2.
 Needs a B200."""
@@ -156,3 +158,26 @@ def test_full_32k_fp32_cancellation_every_element(sat):
     st.close()
     print(f"32K fp32 fsym: worst err/tol = {worst:.3e}")
     assert worst <= 1.0
+
+
+@pytest.mark.slow
+def test_64k_chained_8_ranks_every_element(sat):
+    """configs[4] through the chained partition in the launch configuration bench.chain_projection times:
+    65536 x 65536 int32 cut into 8 strips of 8192 rows, the 8 ranks emulated in one process (Chain.local,
+    inbox pushes into the same HBM), each rank's kernel on the whole GPU in rank order, in place; then every
+    element vs the streaming oracle."""
+    n, N, seed = 65536, 8, 1447
+    x = torch.empty((n, n), dtype=torch.int32, device="cuda")
+    satgen.fill_tensor(x, seed, "u32")
+    h = n // N
+    chains = sat.Chain.local(N, n)
+    try:
+        for r in range(N):
+            sat.sat_chained(x[r * h:(r + 1) * h], out=x[r * h:(r + 1) * h], chain=chains[r])
+        torch.cuda.synchronize()
+    finally:
+        for c in chains:
+            c.close()
+    st = oracle.Stream(n)
+    _compare_rows(x, st, seed, "u32", 0, n, n, 256)
+    st.close()
