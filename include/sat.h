@@ -279,10 +279,13 @@ sat_status_t sat_query_plan(sat_dtype_t dtype, int64_t rows, int64_t cols, int64
 
 /* TEST / TUNING HOOKS (process-wide; for sweeps and tests -- not part of the computing API).
  * variant: -1 = automatic choice, else an index < sat_num_variants() (the shipped library has the
- * four variants auto-selection uses: 0 classic 64x128, 1 TMEM-parked 128x128, 2 u8 integral images,
- * 3 TMEM-parked flat 64x256; -DSAT_EXPERIMENTAL builds append the unshipped tuning configurations);
- * order: 0 = diagonal-major (Fig. 9), 1 = row-major, (g << 8) = diagonal-major over g-tile
- * groups; ctas_per_sm: 0 = occupancy maximum.  Returns INVALID_VALUE for an unknown variant. */
+ * variants auto-selection uses: 0 classic 64x128, 1 TMEM-parked 128x128 with two row walkers,
+ * 2 u8 integral images on 128x128, 3 TMEM-parked flat 64x256, 4 chained strips (sat_compute_chained
+ * only; ignored by sat_compute), 5 u8 integral images on flat 64x256; -DSAT_EXPERIMENTAL builds append
+ * the unshipped tuning configurations); order: 0 = diagonal-major (Fig. 9), 1 = row-major,
+ * 2 = column-major, (g << 8) = diagonal-major over g-wide tile groups, 3 | (g << 8) = diagonal-major
+ * over g-tall groups (the chained strips' order); ctas_per_sm: 0 = occupancy maximum.  Returns
+ * INVALID_VALUE for an unknown variant or order. */
 sat_status_t sat_set_tuning(int variant, int order, int ctas_per_sm);
 int sat_num_variants(void);
 /* Cap the total number of persistent CTAs (0 = no cap).  A cap of 1 runs the whole matrix on one
