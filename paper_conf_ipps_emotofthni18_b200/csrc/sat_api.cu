@@ -312,14 +312,20 @@ int auto_variant(int64_t rows, int64_t cols) {
 // longer waits on the compute warps' stage release.  Measured on the flat 64 x 256 kernel at 32K^2
 // (tools/gpu_r02c.sh, profiles/r02_sweep_prefetch.jsonl): fp32 1.417 -> 1.384 ms, int32 1.409 -> 1.378 ms;
 // with a tile ring of 8 it over-fetches (1.50 ms).  It pays at every size (profiles/r02_sweep_prefetch_sizes.jsonl:
-// 4K^2 40.9 -> 36.7 us, 8K^2 108 -> 102 us, 64K^2 5.55 -> 5.48 ms).  Default: on for the TMEM-parked kernels
-// (the classic kernel has no tile ring); SAT_L2_PREFETCH=0/1 (read once) forces it off / on (tuning switch).
+// 4K^2 40.9 -> 36.7 us, 8K^2 108 -> 102 us, 64K^2 5.55 -> 5.48 ms).  Marking the prefetched lines evict_last
+// (mode 2) keeps them in L2 until their TMA load (which reads them evict_first): 32K^2 fp32 1.383 -> 1.355 ms,
+// int32 1.378 -> 1.351 ms, 16K^2 0.374 -> 0.365 ms, 64K^2 5.48 -> 5.37 ms, chained strip 0.741 -> 0.715 ms per rank;
+// on the 128 x 128 kernel at 4K^2 / 8K^2 it costs 1-3% (tools/gpu_pf.sh).  Default: evict_last for the flat,
+// chained and flat-u8 kernels, plain for the 128 x 128 ones, none for the classic kernel (no tile ring);
+// SAT_L2_PREFETCH=0/1/2 (read once) forces off / plain / evict_last (tuning switch).
 int l2_prefetch_mode(int vi) {
     static const int mode = [] {
         const char* e = std::getenv("SAT_L2_PREFETCH");
         return e ? std::atoi(e) : -1;
     }();
-    return mode >= 0 ? mode : (variants()[vi].family == 2 ? 1 : 0);
+    if (mode >= 0) return mode;
+    if (variants()[vi].family != 2) return 0;
+    return (vi == kVarFlat || vi == kVarChain || vi == kVarU8Flat) ? 2 : 1;
 }
 
 int auto_order(int vi, int64_t cols) {

@@ -214,6 +214,12 @@ __device__ __forceinline__ void bulk_load_1d(void* smem_dst, const void* src, ui
 __device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int x, int y) {
     asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global [%0, {%1, %2}];" ::"l"(map), "r"(x), "r"(y) : "memory");
 }
+// ... with an L2 eviction-priority hint for the prefetched lines
+__device__ __forceinline__ void tma_prefetch_2d_hint(const CUtensorMap* map, int x, int y, uint64_t policy) {
+    asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.L2::cache_hint [%0, {%1, %2}], %3;" ::"l"(map), "r"(x),
+                 "r"(y), "l"(policy)
+                 : "memory");
+}
 
 // 2-D tile shared -> global; out-of-bounds box elements are not written (edge tiles, pitch pad).
 __device__ __forceinline__ void tma_store_2d(const CUtensorMap* map, const void* smem_src, int x, int y) {

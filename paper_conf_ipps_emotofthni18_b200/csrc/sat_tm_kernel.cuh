@@ -1086,8 +1086,15 @@ sat_tm_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_constant_
                 TileInfo ti{t, 0, 0, 0};
                 if (valid) tile_of_serial(t, p.R, p.C, p.order, ti.I, ti.J);
                 if (TMA && valid && p.l2_prefetch) {  // warm L2 while the tile waits for an input stage
+                    if (p.l2_prefetch == 2) {  // tuning: prefetched lines marked evict_last
+                        const uint64_t lpol = policy_evict_last();
 #pragma unroll
-                    for (int bx = 0; bx < Cfg::NB; ++bx) tma_prefetch_2d(&map_in, ti.J * TC + bx * Cfg::TB, ti.I * TR);
+                        for (int bx = 0; bx < Cfg::NB; ++bx)
+                            tma_prefetch_2d_hint(&map_in, ti.J * TC + bx * Cfg::TB, ti.I * TR, lpol);
+                    } else {
+#pragma unroll
+                        for (int bx = 0; bx < Cfg::NB; ++bx) tma_prefetch_2d(&map_in, ti.J * TC + bx * Cfg::TB, ti.I * TR);
+                    }
                 }
                 sm.info[ta.s] = ti;
                 if (!valid) {
