@@ -295,10 +295,21 @@ def main():
     x = x.view(tdt)
     y = torch.empty_like(x)
     comm = chain = None
-    if world > 1 and args.sharded == "gather":
+    fallback = None
+    if world > 1 and args.sharded == "chain":
+        try:
+            chain = sat.Chain(cols)
+        except sat.SatError as e:  # e.g. CUDA IPC between the ranks' GPUs refused: every rank falls back
+            fallback = f"chained strips unavailable ({e}); NCCL gather path"
+        ok = torch.tensor([0 if fallback else 1], dtype=torch.int32, device=dev)
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if int(ok.item()) == 0:
+            if chain is not None:
+                chain.close()
+                chain = None
+            fallback = fallback or "chained strips unavailable on another rank; NCCL gather path"
+    if world > 1 and chain is None:
         comm = sat.Comm()
-    elif world > 1:
-        chain = sat.Chain(cols)
 
     def step():
         if comm is not None:
@@ -378,7 +389,8 @@ def main():
                        "variant": plan["variant"], "order": order_name(plan["order"]),
                        "l2": "inputs (4 B x n^2) larger than the 126 MB L2; no flush",
                        "parallelism": "single GPU" if world == 1 else
-                       f"strips x{world} ({'sat_compute_chained' if chain is not None else 'sat_compute_sharded'})"},
+                       f"strips x{world} ({'sat_compute_chained' if chain is not None else 'sat_compute_sharded'})",
+                       **({"fallback": fallback} if fallback else {})},
             "hbm_gbs": achieved,
             "memcpy": {"ms": memcpy_ms, "gbs": nrows * cols * BYTES_PER_ELEM / (memcpy_ms / 1e3) / 1e9,
                        "overhead_pct": (ms - memcpy_ms) / memcpy_ms * 100.0, "ratio": ms / memcpy_ms,
