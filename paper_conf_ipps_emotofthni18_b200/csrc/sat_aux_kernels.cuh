@@ -86,39 +86,34 @@ __global__ void colsum_reduce_kernel(const V* __restrict__ partial, V* __restric
 }
 
 // Carry row of `rank`: C[j] = sum_{g<rank} gathered[g][j] (ascending g), carry = inclusive
-// row-wise prefix of C.  One CTA of 1024 threads; thread t owns a contiguous chunk.
+// row-wise prefix of C.  One CTA of 1024 threads walking the columns in blocks of 1024: thread t
+// sums column base + t over the lower ranks (coalesced loads), a block scan (warp scans + a scan of the
+// 32 warp totals) gives the in-block prefix, and a running offset carries it across blocks.
 template <typename V>
 __global__ void __launch_bounds__(1024) carry_prefix_kernel(const V* __restrict__ gathered, int rank, int64_t cols,
                                                              V* __restrict__ carry) {
     __shared__ V warp_tot[32];
+    __shared__ V block_tot;
     const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
-    const int64_t chunk = (cols + 1023) / 1024;
-    const int64_t j0 = t * chunk;
-    int64_t j1 = j0 + chunk;
-    if (j1 > cols) j1 = cols;
-    auto C = [&](int64_t j) {
+    V offset = V(0);  // sum of C over all earlier blocks (same value in every thread)
+    for (int64_t base = 0; base < cols; base += 1024) {
+        const int64_t j = base + t;
         V c = V(0);
-        for (int g = 0; g < rank; ++g) c = c + gathered[static_cast<int64_t>(g) * cols + j];
-        return c;
-    };
-    V mine = V(0);
-    for (int64_t j = j0; j < j1; ++j) mine = mine + C(j);
-    // block exclusive scan of the chunk totals (warp scan, then scan of warp totals)
-    V incl = warp_inclusive_scan(mine, lane);
-    if (lane == 31) warp_tot[warp] = incl;
-    __syncthreads();
-    if (warp == 0) {
-        V x = warp_tot[lane];
-        x = warp_inclusive_scan(x, lane);
-        warp_tot[lane] = x;
-    }
-    __syncthreads();
-    const V up = __shfl_up_sync(kFull, incl, 1);
-    V run = (lane == 0) ? V(0) : up;  // exclusive prefix within the warp
-    if (warp > 0) run = warp_tot[warp - 1] + run;
-    for (int64_t j = j0; j < j1; ++j) {
-        run = run + C(j);
-        carry[j] = run;
+        if (j < cols)
+            for (int g = 0; g < rank; ++g) c = c + gathered[static_cast<int64_t>(g) * cols + j];
+        const V incl = warp_inclusive_scan(c, lane);
+        if (lane == 31) warp_tot[warp] = incl;
+        __syncthreads();
+        if (warp == 0) {
+            const V x = warp_inclusive_scan(warp_tot[lane], lane);
+            warp_tot[lane] = x;
+            if (lane == 31) block_tot = x;
+        }
+        __syncthreads();
+        const V pre = warp > 0 ? warp_tot[warp - 1] : V(0);
+        if (j < cols) carry[j] = offset + (pre + incl);
+        offset = offset + block_tot;
+        __syncthreads();  // warp_tot / block_tot are rewritten by the next block
     }
 }
 
