@@ -145,13 +145,14 @@ __global__ void __launch_bounds__(kBoxThreads) box_sum_smem_kernel(const V* __re
 // gridDim.y row bands of H output rows, one block each, sized by the host so the grid is one full wave
 // (blocks = SMs x resident blocks per SM).  A block walks its band top to bottom; output row i needs the
 // SAT row segments d = min(i + rh, rows - 1) and u = i - rh - 1 (columns [p0 - rw - 1, p0 + W - 1 + rw]).
-// Thread 0 fetches both with 1-D bulk copies (TMA engine, one instruction per segment, completion on the
+// Warp 0 fetches both with 1-D bulk copies (TMA engine, one instruction per segment, completion on the
 // ring slot's mbarrier), RB output rows per ring slot, AHEAD slots ahead; a thread evaluates its column
 // for the slot's RB rows as RB independent chains with hoisted offsets.  Measured at 32K^2 int32, r = 8
 // (tools/bench_box.py): row-at-a-time variants ran at 1.1-1.5 TB/s (instruction-issue
 // bound: ncu issue slots 68% busy at ~50 instructions per output); <8, 1> at 4 blocks per SM 1.62 ms =
-// 5.3 TB/s of the algorithmic 8 B/elem, with ncu DRAM read + write 1.02x algorithmic (the strided-row
-// staged kernel below reads the SAT twice from DRAM: 12.9 GB for 8.6 GB algorithmic).
+// 5.3 TB/s of the algorithmic 8 B/elem, with ncu DRAM read + write 1.00x algorithmic (the strided-row
+// staged kernel below reads the SAT twice from DRAM: 12.9 GB for 8.6 GB algorithmic); the slot's copies
+// issued by 8 lanes instead of thread 0: 1.547 ms = 5.55 TB/s.
 // Row d is new data (one DRAM read per SAT row and band); row u is the row d of 2 rh + 1 output rows
 // earlier -- an L2 hit while the concurrent bands' working set, bands x (2 rh + 1) rows x cols x 4 B, fits
 // in L2 (32K columns, rh = 64, two bands: 33 MB of 126 MB).  All blocks walk rows top-down at about the
@@ -196,29 +197,36 @@ __global__ void __launch_bounds__(256) box_band_kernel(const V* __restrict__ b, 
     fence_proxy_async_smem();  // the zeros (generic proxy) before the bulk copies (async proxy)
     __syncthreads();
     const int nslots = (i1 - i0 + RB - 1) / RB;
-    auto issue_slot = [&](int n, int slot) {  // thread 0: segments of output rows i0 + n*RB .. + RB - 1
+    // warp 0: segments of output rows i0 + n*RB .. + RB - 1, lane k < RB issuing row k's copies (the copies
+    // of a slot go out in parallel instead of one after another from a single thread)
+    auto issue_slot = [&](int n, int slot) {
         if (n >= nslots) return;
         const int ia = i0 + n * RB, ib = ia + RB < i1 ? ia + RB : i1;
-        uint32_t bytes = 0;
-        for (int i = ia; i < ib; ++i) bytes += (i - rh - 1 >= 0) ? 2 * seg_bytes : seg_bytes;
-        mbar_arrive_expect_tx(&full[slot], bytes);
-        for (int i = ia; i < ib; ++i) {
+        const int lane = threadIdx.x & 31;
+        if (lane == 0) {
+            uint32_t bytes = 0;
+            for (int i = ia; i < ib; ++i) bytes += (i - rh - 1 >= 0) ? 2 * seg_bytes : seg_bytes;
+            mbar_arrive_expect_tx(&full[slot], bytes);
+        }
+        __syncwarp();
+        const int i = ia + lane;
+        if (lane < RB && i < ib) {
             const int d = i + rh < rows - 1 ? i + rh : rows - 1, u = i - rh - 1;
-            V* sd = ringD + (slot * RB + (i - ia)) * segw + seg_off;
+            V* sd = ringD + (slot * RB + lane) * segw + seg_off;
             bulk_load_1d(sd, b + static_cast<int64_t>(d) * pitch + lo_c, seg_bytes, &full[slot]);
             if (u >= 0)
-                bulk_load_1d(ringU + (slot * RB + (i - ia)) * segw + seg_off, b + static_cast<int64_t>(u) * pitch + lo_c,
+                bulk_load_1d(ringU + (slot * RB + lane) * segw + seg_off, b + static_cast<int64_t>(u) * pitch + lo_c,
                              seg_bytes, &full[slot]);
         }
     };
-    if (threadIdx.x == 0)
+    if (threadIdx.x < 32)
         for (int n = 0; n < kBandAhead; ++n) issue_slot(n, n);
     const int64_t jcol = p0 + threadIdx.x;  // the fast path's column of this thread
     const int kr0 = static_cast<int>((jcol + rw < hi ? jcol + rw : hi) - a0), kl0 = static_cast<int>(jcol - rw - 1 - a0);
     int slot = 0;
     uint32_t phase = 0;
     for (int n = 0; n < nslots; ++n) {
-        if (threadIdx.x == 0) {  // that slot was last read for slot number n + kBandAhead - Q = n - 2 (barrier below)
+        if (threadIdx.x < 32) {  // that slot was last read for slot number n + kBandAhead - Q = n - 2 (barrier below)
             const int f = slot + kBandAhead < Q ? slot + kBandAhead : slot + kBandAhead - Q;
             issue_slot(n + kBandAhead, f);
         }
