@@ -381,6 +381,33 @@ def test_host_pipeline(sat, dist):
         assert_f32_tol(np.ascontiguousarray(view), b)
 
 
+def test_host_pipeline_concurrent_threads(sat):
+    """sat_compute_host from several host threads at once (its per-device staging lock): every
+    call's result stays its own.  Sizes differ so that a later call also regrows the staging buffer."""
+    import threading
+
+    shapes = [(3000, 2500), (5000, 2100), (1200, 4100), (4100, 3000)]
+    inputs = [satgen.gen_host(r, c, seed=700 + k, dist="u32") for k, (r, c) in enumerate(shapes)]
+    outs = [None] * len(shapes)
+    errs = []
+
+    def run(k):
+        try:
+            for _ in range(3):
+                outs[k] = sat.sat_host(inputs[k])
+        except Exception as e:  # pragma: no cover - reported below
+            errs.append(e)
+
+    threads = [threading.Thread(target=run, args=(k,)) for k in range(len(shapes))]
+    for t in threads:
+        t.start()
+    for t in threads:
+        t.join(timeout=300)
+    assert not errs, errs
+    for k, a in enumerate(inputs):
+        assert (outs[k] == oracle.sat_i32(a)).all(), k
+
+
 # ----------------------------------------------------------------------------------- tile order (Fig. 9)
 @pytest.mark.parametrize("R,C", [(5, 5), (1, 9), (7, 1), (4, 11), (13, 3), (64, 64), (256, 512)])
 def test_device_tile_order_matches_fig9_order(sat, R, C):
