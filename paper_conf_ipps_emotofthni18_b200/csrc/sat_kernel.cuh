@@ -30,6 +30,22 @@
 
 namespace sat {
 
+// Diagnosis builds only (-DSAT_DIAG_SITE=k): a per-THREAD pseudo-random sleep at publication site k
+#if defined(SAT_DIAG_SITE)
+#define SAT_DIAG_SLEEP(site)                                                                                   \
+    do {                                                                                                      \
+        if ((site) == SAT_DIAG_SITE) {                                                                        \
+            uint64_t z_ = static_cast<uint64_t>(clock64()) ^ (static_cast<uint64_t>(blockIdx.x) << 40) ^      \
+                          (static_cast<uint64_t>(threadIdx.x) << 20);                                         \
+            z_ = (z_ ^ (z_ >> 30)) * 0xbf58476d1ce4e5b9ull;                                                   \
+            z_ ^= z_ >> 31;                                                                                   \
+            if ((z_ & 3u) == 0u) __nanosleep(static_cast<unsigned>((z_ >> 8) & 4095u));                      \
+        }                                                                                                     \
+    } while (0)
+#else
+#define SAT_DIAG_SLEEP(site) (void)0
+#endif
+
 constexpr uint32_t kLocal = 1u;
 constexpr uint32_t kIncl = 2u;
 constexpr uint32_t kEpochMax = (1u << 30) - 1u;
@@ -470,6 +486,7 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
         //      Row slots: lane 31 of every warp (last column of its rows); column slots: the last
         //      warp (bottom row).  Edge tiles publish inclusive at once (their carry is zero).
         if (lane == 31) {
+            SAT_DIAG_SLEEP(1);
             uint64_t* rs = p.row_slots + tidx * TR + row0;
             const uint32_t kind = (J == 0) ? kIncl : kLocal;
 #pragma unroll
@@ -484,6 +501,7 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
         if (warp == NW - 1) {
             uint64_t* cs = p.col_slots + tidx * TC + col0;
             const uint32_t kind = (I == 0) ? kIncl : kLocal;
+            SAT_DIAG_SLEEP(2);
             st_relaxed2(cs, pack(epoch, kind, to_bits(v[RPW - 1][0])), pack(epoch, kind, to_bits(v[RPW - 1][1])));
             st_relaxed2(cs + 2, pack(epoch, kind, to_bits(v[RPW - 1][2])), pack(epoch, kind, to_bits(v[RPW - 1][3])));
             if (lane == 31) sm.total = v[RPW - 1][3];
@@ -535,6 +553,7 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
         SAT_JITTER_WARP();
         // ---- Steps 2.A.3 / 2.B.3: publish the inclusive aggregates (owners of the local values)
         if (lane == 31 && J > 0) {
+            SAT_DIAG_SLEEP(5);
             uint64_t* rs = p.row_slots + tidx * TR + row0;
 #pragma unroll
             for (int r = 0; r < RPW; r += 2) {
@@ -547,6 +566,7 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
             }
         }
         if (warp == NW - 1 && I > 0) {
+            SAT_DIAG_SLEEP(6);
             uint64_t* cs = p.col_slots + tidx * TC + col0;
             const uint4 q = *reinterpret_cast<const uint4*>(&sm.cp[col0]);
             st_relaxed2(cs, pack(epoch, kIncl, to_bits(v[RPW - 1][0] + from_bits<V>(q.x))),
@@ -560,7 +580,10 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
         uint64_t* cslot = p.corner_slots + tidx;
         if (!sm.corner_ok) {  // uniform: read after barrier (3)
             if (warp == 2) {
-                if (lane == 0) st_relaxed(cslot, pack(epoch, kLocal, to_bits(gls)));
+                if (lane == 0) {
+                    SAT_DIAG_SLEEP(3);
+                    st_relaxed(cslot, pack(epoch, kLocal, to_bits(gls)));
+                }
                 V corner;
                 lookback_diag<V>(p.corner_slots, I, J, p.C, epoch, /*blocking=*/true, lane,
                                  diag_word(p.corner_slots, I, J, p.C, 1 + lane), corner);
@@ -569,7 +592,10 @@ sat_tiles_kernel(const __grid_constant__ CUtensorMap map_in, const __grid_consta
             __syncthreads();  // (4) corner visible (rare)
         }
         const V corner = sm.corner;
-        if (warp == 2 && lane == 0) st_relaxed(cslot, pack(epoch, kIncl, to_bits(corner + gls)));
+        if (warp == 2 && lane == 0) {
+            SAT_DIAG_SLEEP(4);
+            st_relaxed(cslot, pack(epoch, kIncl, to_bits(corner + gls)));
+        }
         SAT_CLK(c_b4);
         SAT_ST(kStDiagLate, c_b4 - c_b3b);
 
