@@ -73,7 +73,11 @@ typedef struct sat_comm_s* sat_comm_t;
 sat_status_t sat_compute_i32(const int32_t* src, int32_t* dst, int64_t rows, int64_t cols,
                              int64_t pitch, void* stream);
 
-/* SAT of an fp32 matrix (the paper's "4-byte float"); tolerance rule above. */
+/* SAT of an fp32 matrix (the paper's "4-byte float"); tolerance rule above.
+ * CUDA graphs: after one call on a stream (which creates that stream's workspace), calls on that stream
+ * are capturable and replayable -- the launch epoch lives on the device, nothing synchronises the host --
+ * as long as no captured call needs a larger workspace than the calls made before capture
+ * (tests/test_gpu_batched.py::test_sat_calls_replay_from_a_cuda_graph). */
 sat_status_t sat_compute_f32(const float* src, float* dst, int64_t rows, int64_t cols,
                              int64_t pitch, void* stream);
 

@@ -206,3 +206,32 @@ def test_batched_u8_matches_single(sat):
     got = run_u8(sat, img)
     for k in range(3):
         assert (sat.sat_u8(torch.from_numpy(img[k].copy()).cuda()).cpu().numpy() == got[k]).all()
+
+
+def test_sat_calls_replay_from_a_cuda_graph():
+    """Small matrices are launch-latency bound (NEXT-2): after one warm-up call on a stream (which
+    creates that stream's workspace), sat_compute is capturable -- epochs advance on the device, no host
+    sync -- so a CUDA graph of many calls replays with exact results every time."""
+    import paper_conf_ipps_emotofthni18_b200 as sat
+
+    shapes = [(256, 256), (300, 517), (1024, 1024), (64, 2000)]
+    xs = [torch.from_numpy(satgen.gen_host(r, c, seed=900 + r, dist="u32")).cuda() for r, c in shapes]
+    ys = [torch.empty_like(x) for x in xs]
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        for x, y in zip(xs, ys):
+            sat.sat(x, out=y, stream=s)  # warm-up: workspace, occupancy caches
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for _ in range(3):
+            for x, y in zip(xs, ys):
+                sat.sat(x, out=y, stream=s)
+    for _ in range(5):
+        for y in ys:
+            y.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        for x, y in zip(xs, ys):
+            assert (y.cpu().numpy() == oracle.sat_i32(x.cpu().numpy())).all()
