@@ -137,3 +137,21 @@ def test_batched_binding_rejects_bad_tensors(sat):
         sat.sat_batched(torch.zeros(2, 3, 4, dtype=torch.int32))  # not a CUDA tensor
     with pytest.raises(ValueError):
         sat.sat_batched_u8(torch.zeros(2, 3, 4, dtype=torch.uint8))
+
+
+def test_wide_argument_validation_without_gpu(sat):
+    """sat_compute_f32_f64 / sat_compute_moments_f32 reject bad arguments before any CUDA call."""
+    from paper_conf_ipps_emotofthni18_b200 import _lib
+
+    L = _lib.lib()
+    for F in (L.sat_compute_f32_f64, L.sat_compute_moments_f32):
+        assert F(None, 5, None, 5, 0, 5, None) == 0  # empty: no-op, null pointers allowed
+        assert F(None, 5, None, 5, 4, 0, None) == 0
+        assert F(1 << 20, 4, 1 << 21, 5, 4, 5, None) == 1  # src_pitch < cols
+        assert F(1 << 20, 5, 1 << 21, 4, 4, 5, None) == 1  # dst_pitch < cols
+        assert F(1 << 20, 5, 1 << 21, 5, -1, 5, None) == 1  # negative rows
+        assert F(None, 5, 1 << 21, 5, 4, 5, None) == 1  # null src
+        assert F((1 << 20) + 2, 5, 1 << 21, 5, 4, 5, None) == 2  # src not 4-byte aligned
+        assert F(1 << 20, 5, (1 << 21) + 4, 5, 4, 5, None) == 2  # dst not 8-byte aligned
+        assert F(1 << 20, 5, (1 << 20) + 8, 5, 4, 5, None) == 1  # overlap
+        assert b"overlap" in L.sat_last_error_detail()
