@@ -227,14 +227,14 @@ sat_status_t sat_compute_sharded(sat_comm_t comm, sat_dtype_t dtype, const void*
  *
  * The same horizontal strip partition as sat_compute_sharded (rank r holds global rows
  * [row0_r, row0_r + strip_rows)), computed in ONE pass per rank: each element is read once and written
- * once (2 accesses instead of the 3 of colsum + all-gather + SAT).  A rank walks its strip in
- * column-major tile order; as soon as its bottom tile of tile column J has resolved the strip's column
- * sums over J (Step 2.B of P:198-202 restricted to the strip), its kernel pushes them -- as epoch-tagged
- * 64-bit status words, the single-copy-atomic protocol of the look-back (R11) -- straight
- * into the inbox of every downstream rank through peer-mapped memory over NVLink (CUDA IPC); a
- * downstream rank's column walker adds the upstream column sums of rank 0..r-1 (ascending) to its
- * strip-local column carry.  The column sums of tile column J arrive about one tile column of work
- * after they are needed, well inside the pipeline's parking window, so the ranks run concurrently
+ * once (2 accesses instead of the 3 of colsum + all-gather + SAT).  A rank walks its strip in the
+ * anti-diagonal order of groups of 8 vertically adjacent tiles (Fig. 9's order over tall groups); each
+ * tile's column walker adds the carry T(r-1) -- the column sums of all rows of ranks 0..r-1 over its tile
+ * column -- from the rank's inbox to its strip-local column carry, and as soon as the bottom tile of tile
+ * column J has resolved, the kernel pushes T(r) = its strip column sums + T(r-1) -- as epoch-tagged 64-bit
+ * status words, the single-copy-atomic protocol of the look-back (R11) -- into the inbox of
+ * rank r+1 only, through peer-mapped memory over NVLink (CUDA IPC).  Every rank polls one vector and pushes
+ * one per tile column, whatever nranks; a rank lags the one above by ~1/8 of its strip's tile rows
  * (DESIGN.md Sec. 7).  No NCCL call on the data path.
  *
  * Setup (collective, once per partition): every rank calls sat_chain_create on its own device,
